@@ -1,0 +1,161 @@
+"""CPU oracle for libbulkgcd -- TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+``--impl reference`` legs may import this package.  The product path
+(paper_conf_ipps_fujitani15_b200, include/bulkgcd.h) never imports it and the
+two share no code; only the seeded input generators in ``synth`` serve both.
+
+* :mod:`oracle.gcd_oracle` (C, ``gcd_oracle.c``): the definition -- the
+  Original Euclidean algorithm (§II) over schoolbook bignums with
+  Knuth Algorithm D division (paper ref. [15]).  Exact gcd of any operands.
+* :mod:`oracle.approx_model` (Python ints): the paper's Approximate Euclidean
+  algorithm step by step (L107, L127, L255), d-generic, with counters; used to
+  pin the worked examples (Table III, the approx examples) and Table IV, and
+  for per-pair iteration-count parity with the GPU.
+* :func:`rsa_hit` -- the RSA-mode result mapping.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+from . import approx_model  # noqa: F401  (re-exported)
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "gcd_oracle.c")
+_SO = os.path.join(_HERE, "libgcd_oracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile the C oracle (gcc -O2) -> oracle/libgcd_oracle.so."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        tmp = _SO + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-shared", "-fPIC", "-o", tmp, _SRC, "-lpthread"])
+        os.replace(tmp, _SO)
+    return _SO
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        lib = ctypes.CDLL(build())
+        vp, u32, sz = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_size_t
+        lib.oracle_gcd.argtypes = [vp, vp, u32, vp]
+        lib.oracle_gcd.restype = ctypes.c_long
+        lib.oracle_gcd_trace.argtypes = [vp, vp, u32, vp, vp, ctypes.c_long]
+        lib.oracle_gcd_trace.restype = ctypes.c_long
+        lib.oracle_divmod.argtypes = [vp, vp, u32, vp, vp]
+        lib.oracle_divmod.restype = ctypes.c_int
+        lib.oracle_gcd_batch.argtypes = [vp, vp, sz, u32, vp, ctypes.c_int]
+        lib.oracle_gcd_batch.restype = ctypes.c_int
+        lib.oracle_gcd_index_pairs.argtypes = [vp, vp, vp, sz, u32, vp, ctypes.c_int]
+        lib.oracle_gcd_index_pairs.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+def _limbs(x: int, n: int) -> np.ndarray:
+    return np.frombuffer(int(x).to_bytes(4 * n, "little"), dtype="<u4").astype(np.uint32)
+
+
+def _int(a: np.ndarray) -> int:
+    return int.from_bytes(np.ascontiguousarray(a, dtype="<u4").tobytes(), "little")
+
+
+def _nlimbs(*xs: int) -> int:
+    return max(1, max((x.bit_length() + 31) // 32 for x in xs))
+
+
+def gcd(a: int, b: int) -> int:
+    """Exact gcd of two non-negative Python ints through the C oracle."""
+    n = _nlimbs(a, b)
+    A, B, G = _limbs(a, n), _limbs(b, n), np.zeros(n, np.uint32)
+    if _load().oracle_gcd(A.ctypes.data, B.ctypes.data, n, G.ctypes.data) < 0:
+        raise ValueError("operand too large for the oracle")
+    return _int(G)
+
+
+def gcd_trace(a: int, b: int, qmax: int = 4096) -> tuple[int, int, list[int]]:
+    """(gcd, iterations, quotients) of the Original Euclidean algorithm (L55)."""
+    n = _nlimbs(a, b)
+    A, B, G = _limbs(a, n), _limbs(b, n), np.zeros(n, np.uint32)
+    Q = np.zeros(qmax, np.uint64)
+    it = _load().oracle_gcd_trace(A.ctypes.data, B.ctypes.data, n, G.ctypes.data, Q.ctypes.data, qmax)
+    if it < 0:
+        raise ValueError("operand too large for the oracle")
+    return _int(G), int(it), [int(q) for q in Q[:min(it, qmax)]]
+
+
+def divmod_(x: int, y: int) -> tuple[int, int]:
+    """(x div y, x mod y) via Knuth Algorithm D (the oracle's division)."""
+    n = _nlimbs(x, y)
+    X, Y = _limbs(x, n), _limbs(y, n)
+    Q, R = np.zeros(n, np.uint32), np.zeros(n, np.uint32)
+    if _load().oracle_divmod(X.ctypes.data, Y.ctypes.data, n, Q.ctypes.data, R.ctypes.data) != 0:
+        raise ZeroDivisionError
+    return _int(Q), _int(R)
+
+
+def gcd_batch(A: np.ndarray, B: np.ndarray, nthreads: int | None = None) -> np.ndarray:
+    """G[k] = gcd(A[k], B[k]) for uint32[m, W] row-major limb arrays."""
+    A = np.ascontiguousarray(A, dtype=np.uint32)
+    B = np.ascontiguousarray(B, dtype=np.uint32)
+    assert A.shape == B.shape and A.ndim == 2
+    G = np.zeros_like(A)
+    nt = nthreads or os.cpu_count() or 1
+    if A.shape[0] and _load().oracle_gcd_batch(A.ctypes.data, B.ctypes.data, A.shape[0], A.shape[1],
+                                               G.ctypes.data, nt) != 0:
+        raise RuntimeError("oracle_gcd_batch failed")
+    return G
+
+
+def gcd_index_pairs(N: np.ndarray, ii, jj, nthreads: int | None = None) -> np.ndarray:
+    """G[k] = gcd(N[ii[k]], N[jj[k]])."""
+    N = np.ascontiguousarray(N, dtype=np.uint32)
+    ii = np.ascontiguousarray(ii, dtype=np.uint64)
+    jj = np.ascontiguousarray(jj, dtype=np.uint64)
+    G = np.zeros((ii.size, N.shape[1]), np.uint32)
+    nt = nthreads or os.cpu_count() or 1
+    if ii.size and _load().oracle_gcd_index_pairs(N.ctypes.data, ii.ctypes.data, jj.ctypes.data, ii.size,
+                                                  N.shape[1], G.ctypes.data, nt) != 0:
+        raise RuntimeError("oracle_gcd_index_pairs failed")
+    return G
+
+
+def bitlen_rows(G: np.ndarray) -> np.ndarray:
+    """Bit length of each row of a uint32[m, W] limb array."""
+    G = np.asarray(G, dtype=np.uint32)
+    nz = G != 0
+    top = np.where(nz.any(axis=1), G.shape[1] - 1 - np.argmax(nz[:, ::-1], axis=1), -1)
+    word = G[np.arange(G.shape[0]), np.maximum(top, 0)].astype(np.uint64)
+    wbits = np.zeros(G.shape[0], np.int64)
+    w = word.copy()
+    while np.any(w):
+        wbits += (w != 0)
+        w >>= np.uint64(1)
+    return np.where(top >= 0, top * 32 + wbits, 0)
+
+
+def rsa_hit(g_bitlen, bits: int):
+    """RSA-mode mapping: the early-terminated
+    algorithm reports g iff g has at least s/2 bits, otherwise "coprime" (1)."""
+    return np.asarray(g_bitlen) >= bits // 2
+
+
+def all_pairs_hits(N: np.ndarray, bits: int, ii=None, jj=None, nthreads: int | None = None):
+    """RSA-mode hit set over the given (i<j) pairs (default: every pair).
+
+    Returns a sorted list of (i, j, g_int) with bitlen(g) >= bits/2.
+    """
+    n = N.shape[0]
+    if ii is None:
+        ii, jj = np.triu_indices(n, k=1)
+    G = gcd_index_pairs(N, ii, jj, nthreads)
+    hit = rsa_hit(bitlen_rows(G), bits)
+    out = [(int(ii[k]), int(jj[k]), _int(G[k])) for k in np.nonzero(hit)[0]]
+    out.sort()
+    return out

@@ -1,0 +1,138 @@
+"""Pins for the CPU model of the paper's Approximate Euclidean algorithm
+(oracle/approx_model.py): the worked examples (Table III, the approx()
+examples, Table II's Fast Euclid column), Table IV's mean iteration counts, the
+quotient bound alpha*D^beta <= X div Y (L123), and agreement with math.gcd."""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from conftest import read_golden
+from oracle import approx_model as am
+
+
+def test_approx_examples():
+    for X, Y, a, b, case, _cite in read_golden("approx_examples.txt"):
+        assert am.approx(int(X), int(Y), 4) == (int(a), int(b), case)
+
+
+def test_table3_trace():
+    rows = read_golden("table3_approx_euclid.txt")
+    head = {r[0]: r[1] for r in rows[:4]}
+    t = am.approximate_euclid(int(head["X"], 16), int(head["Y"], 16), d=int(head["d"]), record=True, check=True)
+    steps = rows[4:]
+    assert t.iterations == len(steps) == 9
+    assert t.gcd == int(head["gcd"])
+    for got, (_n, case, a, b, x, y) in zip(t.steps, steps):
+        assert got == (case, int(a), int(b), int(x, 16), int(y, 16))
+    assert t.bound_violations == 0
+
+
+def test_table2_fast_euclid():
+    rows = {r[0]: r[1:] for r in read_golden("table2_original_euclid.txt")}
+    g, it, qs = am.fast_euclid(int(rows["X"][0]), int(rows["Y"][0]))
+    assert g == int(rows["gcd"][0])
+    assert it == int(rows["fast_iterations"][0])
+    assert qs == [int(q) for q in rows["fast_quotients"]]
+
+
+def test_fast_binary_special_case():
+    """L111: with (alpha, beta) = (1, 0) always, the algorithm is Fast Binary Euclid;
+    Table I (L47) says Fast Binary takes 16 iterations on the Table I inputs."""
+    X, Y = 1043915, 768955
+    it = 0
+    while Y:
+        X = am.rshift(X - Y)
+        if X < Y:
+            X, Y = Y, X
+        it += 1
+    assert (X, it) == (5, 16)
+
+
+@pytest.mark.parametrize("bits", [64, 96, 128, 256, 1024])
+def test_exact_mode_matches_math_gcd(bits):
+    A, B = synth.mixed_pairs(440, bits, seed=100 + bits)
+    for a, b in zip(A, B):
+        t = am.gcd_exact(a, b)
+        assert t.gcd == math.gcd(a, b), (a, b)
+
+
+def test_bound_and_iteration_invariants():
+    """alpha*D^beta <= X div Y (L123), alpha < D outside Case 1 (L133, O4.14),
+    <= 2s iterations (L49, L61) on every rare-path category."""
+    bits = 256
+    A, B = synth.mixed_pairs(660, bits, seed=7)
+    for a, b in zip(A, B):
+        if a == 0 or b == 0:
+            continue
+        X, Y = am.rshift(a), am.rshift(b)
+        t = am.approximate_euclid(X, Y, 32, check=True)
+        assert t.bound_violations == 0
+        assert t.iterations <= 2 * bits
+    # Cases 2-4 return alpha < D (sampled directly)
+    rng = np.random.default_rng(8)
+    for _ in range(3000):
+        X = int.from_bytes(rng.bytes(int(rng.integers(9, 40))), "little") | 1
+        Y = int.from_bytes(rng.bytes(int(rng.integers(1, 40))), "little") | 1
+        if X < Y:
+            X, Y = Y, X
+        a, b, case = am.approx(X, Y, 32)
+        assert a * (1 << (32 * b)) <= X // Y
+        assert a >= 1
+        if case != "1":
+            assert a < (1 << 32)
+
+
+def test_rare_paths_exercised():
+    """The mixed generator really reaches beta > 0, rshift >= d and every case."""
+    A, B = synth.mixed_pairs(1100, 1024, seed=9)
+    cases, beta, rge = {}, 0, 0
+    for a, b in zip(A, B):
+        if a == 0 or b == 0:
+            continue
+        t = am.gcd_exact(a, b)
+        beta += t.beta_pos
+        rge += t.r_ge_d
+        for k, v in t.cases.items():
+            cases[k] = cases.get(k, 0) + v
+    assert beta > 0 and rge > 0
+    assert set(cases) >= {"1", "2-A", "2-B", "3-A", "3-B", "4-A", "4-B", "4-C"}
+
+
+def test_rsa_mode_semantics(cfg1):
+    """Early termination returns g iff bitlen(g) >= s/2 (O3), matching the oracle's
+    exact gcd under the same mapping, and finds exactly the planted hits."""
+    N = synth.ints(cfg1.N)
+    hits = []
+    for i in range(len(N)):
+        for j in range(i + 1, len(N)):
+            t = am.gcd_rsa(N[i], N[j], 1024)
+            if t.gcd != 1:
+                hits.append((i, j, t.gcd))
+    assert hits == cfg1.truth
+
+
+def _table4():
+    return {(r[0], int(r[1])): [float(x) for x in r[2:]] for r in read_golden("table4_iterations.txt")}
+
+
+@pytest.mark.parametrize("bits,npairs", [(512, 3000), (1024, 3000), (2048, 400)])
+def test_table4_means(bits, npairs):
+    """Table IV column (E) (and (A) via the oracle) within 3 combined standard
+    errors of the paper's 10,000-pair means.  Inputs: synthetic OpenSSL-style moduli."""
+    tab = _table4()
+    ms = synth.moduli(npairs + 1, bits, seed=4000 + bits)
+    N = synth.ints(ms.N)
+    early = np.array([am.gcd_rsa(N[k], N[k + 1], bits).iterations for k in range(npairs)], float)
+    non = np.array([am.approximate_euclid(N[k], N[k + 1], 32).iterations for k in range(min(npairs, 1000))],
+                   float)
+    for name, arr, paper in (("early", early, tab[("early", bits)][4]), ("nonterm", non, tab[("nonterm", bits)][4])):
+        se = math.sqrt(arr.var() / arr.size + arr.var() / 10000)
+        assert abs(arr.mean() - paper) <= 3 * se + 0.05, (name, bits, arr.mean(), paper, se)
+    # column (A): the Original Euclidean algorithm's iteration count, from the C oracle
+    orig = np.array([oracle.gcd_trace(N[k], N[k + 1], qmax=1)[1] for k in range(min(npairs, 1000))], float)
+    paper_a = tab[("nonterm", bits)][0]
+    se = math.sqrt(orig.var() / orig.size + orig.var() / 10000)
+    assert abs(orig.mean() - paper_a) <= 3 * se + 0.05, (bits, orig.mean(), paper_a)
