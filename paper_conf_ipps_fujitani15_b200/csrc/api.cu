@@ -1,0 +1,335 @@
+// api.cu -- host side of libbulkgcd: the C ABI of include/bulkgcd.h.
+//
+// Validation, stream-ordered device buffers, layout transforms, kernel
+// launches (persistent grids sized to the SM count), hit-buffer overflow
+// retry and the final (i, j) sort.  No compute happens on the host.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <numeric>
+#include <vector>
+
+#include "../../include/bulkgcd.h"
+#include "kernels.cuh"
+
+using namespace bulkgcd;
+
+namespace {
+
+thread_local char g_err[512] = "";
+
+int set_err(int code, const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof g_err, fmt, ap);
+    va_end(ap);
+    return code;
+}
+
+#define CK(call)                                                                                   \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess) {                                                                   \
+            int code_ = (e_ == cudaErrorMemoryAllocation) ? BULKGCD_ENOMEM : BULKGCD_ECUDA;        \
+            return set_err(code_, "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_)); \
+        }                                                                                          \
+    } while (0)
+
+int words_for(uint32_t bits) {
+    switch (bits) {
+        case 512: return 16;
+        case 1024: return 32;
+        case 2048: return 64;
+        default: return 0;
+    }
+}
+
+int sm_count() {
+    int dev = 0, n = 148;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    return n > 0 ? n : 148;
+}
+
+int device_check() {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return set_err(BULKGCD_ENODEV, "no CUDA device: %s", cudaGetErrorString(e));
+    int major = 0, minor = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+    cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+    if (major != 10 || minor != 0)
+        return set_err(BULKGCD_ENODEV, "device %d is sm_%d%d; libbulkgcd is built for sm_100a only", dev, major,
+                       minor);
+    return 0;
+}
+
+// RAII stream-ordered device buffer.
+struct DBuf {
+    void *p = nullptr;
+    cudaStream_t s = nullptr;
+    DBuf() = default;
+    DBuf(const DBuf &) = delete;
+    ~DBuf() {
+        if (p) cudaFreeAsync(p, s);
+    }
+    cudaError_t alloc(size_t bytes, cudaStream_t st) {
+        s = st;
+        return cudaMallocAsync(&p, bytes ? bytes : 16, st);
+    }
+    template <class T>
+    T *as() const { return (T *)p; }
+};
+
+size_t pad32(size_t m) { return (m + 31) / 32 * 32; }
+
+template <int W>
+int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m, size_t m_pad, int mode,
+                 uint32_t *d_iters, unsigned long long *scratch, unsigned flags, cudaStream_t st) {
+    CK(cudaMemsetAsync(scratch, 0, 4 * sizeof(unsigned long long), st));
+    PairsArgs a{dA, dB, dG, m, m_pad, scratch + 1, d_iters, scratch + 2, W * 16};
+    uint64_t cohorts = (m + 31) / 32;
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * 4, (cohorts + 3) / 4);
+    if (grid == 0) return 0;
+    bool stats = (flags & BULKGCD_FLAG_STATS) || d_iters;
+    if (mode == BULKGCD_MODE_RSA) {
+        if (stats) pairs_kernel<W, true, true><<<(unsigned)grid, THREADS, 0, st>>>(a);
+        else pairs_kernel<W, true, false><<<(unsigned)grid, THREADS, 0, st>>>(a);
+    } else {
+        if (stats) pairs_kernel<W, false, true><<<(unsigned)grid, THREADS, 0, st>>>(a);
+        else pairs_kernel<W, false, false><<<(unsigned)grid, THREADS, 0, st>>>(a);
+    }
+    CK(cudaGetLastError());
+    return 0;
+}
+
+template <int W>
+int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t c0, uint64_t c1, uint32_t *dHits,
+                    uint64_t cap, unsigned long long *counters, unsigned flags, cudaStream_t st) {
+    CK(cudaMemsetAsync(counters, 0, 4 * sizeof(unsigned long long), st));
+    if (c1 <= c0) return 0;
+    AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
+    uint64_t warps = c1 - c0;
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * 4, (warps + 3) / 4);
+    if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, 0, st>>>(a);
+    else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, 0, st>>>(a);
+    CK(cudaGetLastError());
+    return 0;
+}
+
+int check_moduli(const uint32_t *N, size_t n, int W) {
+    for (size_t i = 0; i < n; ++i) {
+        const uint32_t *x = N + i * W;
+        if ((x[0] & 1u) == 0)
+            return set_err(BULKGCD_EINVAL, "modulus %zu is even (RSA mode needs odd moduli > 1)", i);
+        bool gt1 = x[0] > 1;
+        for (int k = 1; k < W && !gt1; ++k) gt1 = x[k] != 0;
+        if (!gt1) return set_err(BULKGCD_EINVAL, "modulus %zu is 1 (RSA mode needs odd moduli > 1)", i);
+    }
+    return 0;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *bulkgcd_strerror(int code) {
+    switch (code) {
+        case BULKGCD_OK: return "ok";
+        case BULKGCD_EINVAL: return "invalid argument";
+        case BULKGCD_ENOMEM: return "out of memory";
+        case BULKGCD_ECUDA: return "CUDA error";
+        case BULKGCD_ENODEV: return "no sm_100 device";
+        default: return "unknown error";
+    }
+}
+
+const char *bulkgcd_last_error(void) { return g_err; }
+
+int bulkgcd_device_check(void) { return device_check(); }
+
+size_t bulkgcd_blocked_words(size_t n, uint32_t bits) { return pad32(n) * (size_t)words_for(bits); }
+
+uint64_t bulkgcd_cohort_count(size_t n) { return cohort_total(n); }
+
+int bulkgcd_interleave(const uint32_t *d_in, uint32_t *d_out, size_t m, size_t m_pad, uint32_t bits,
+                       int to_interleaved, void *stream) {
+    int W = words_for(bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u", bits);
+    if (m_pad < m || m_pad % 32) return set_err(BULKGCD_EINVAL, "m_pad must be >= m and a multiple of 32");
+    if (m_pad == 0) return 0;
+    if (!d_in || !d_out) return set_err(BULKGCD_EINVAL, "null pointer");
+    dim3 grid((unsigned)(m_pad / 32), (unsigned)((W + 31) / 32)), block(32, 8);
+    interleave_kernel<<<grid, block, 0, (cudaStream_t)stream>>>(d_in, d_out, m, m_pad, W, to_interleaved);
+    CK(cudaGetLastError());
+    return 0;
+}
+
+int bulkgcd_layout_blocked(const uint32_t *d_N, uint32_t *d_N_blk, size_t n, uint32_t bits, void *stream) {
+    int W = words_for(bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u", bits);
+    if (n == 0) return 0;
+    if (!d_N || !d_N_blk) return set_err(BULKGCD_EINVAL, "null pointer");
+    dim3 grid((unsigned)(pad32(n) / 32), (unsigned)((W + 31) / 32)), block(32, 8);
+    blocked_kernel<<<grid, block, 0, (cudaStream_t)stream>>>(d_N, d_N_blk, n, W);
+    CK(cudaGetLastError());
+    return 0;
+}
+
+int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G, size_t m, size_t m_pad,
+                         uint32_t bits, int mode, uint32_t *d_iters, unsigned long long *d_scratch, unsigned flags,
+                         void *stream) {
+    int W = words_for(bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u", bits);
+    if (mode != BULKGCD_MODE_EXACT && mode != BULKGCD_MODE_RSA) return set_err(BULKGCD_EINVAL, "bad mode %d", mode);
+    if (m == 0) return 0;
+    if (!d_A || !d_B || !d_G || !d_scratch) return set_err(BULKGCD_EINVAL, "null pointer");
+    if (m_pad < m || m_pad % 32) return set_err(BULKGCD_EINVAL, "m_pad must be >= m and a multiple of 32");
+    cudaStream_t st = (cudaStream_t)stream;
+    switch (W) {
+        case 16: return launch_pairs<16>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
+        case 32: return launch_pairs<32>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
+        default: return launch_pairs<64>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
+    }
+}
+
+int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t n, uint32_t bits,
+                           uint64_t cohort_begin, uint64_t cohort_end, uint32_t *d_hits, uint64_t hit_cap,
+                           unsigned long long *d_counters, unsigned flags, void *stream) {
+    int W = words_for(bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u", bits);
+    if (!d_counters) return set_err(BULKGCD_EINVAL, "null counters");
+    uint64_t total = cohort_total(n);
+    if (cohort_end > total) cohort_end = total;
+    if (cohort_begin > cohort_end) cohort_begin = cohort_end;
+    if (cohort_end > cohort_begin && (!d_N || !d_N_blk)) return set_err(BULKGCD_EINVAL, "null pointer");
+    if (hit_cap && !d_hits) return set_err(BULKGCD_EINVAL, "null hit buffer with hit_cap > 0");
+    cudaStream_t st = (cudaStream_t)stream;
+    switch (W) {
+        case 16: return launch_allpairs<16>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
+        case 32: return launch_allpairs<32>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
+        default: return launch_allpairs<64>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
+    }
+}
+
+int bulkgcd_pairs_ex(const uint32_t *A, const uint32_t *B, size_t m, uint32_t bits, int mode, uint32_t *G,
+                     uint32_t *iters) {
+    int W = words_for(bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048)", bits);
+    if (mode != BULKGCD_MODE_EXACT && mode != BULKGCD_MODE_RSA) return set_err(BULKGCD_EINVAL, "bad mode %d", mode);
+    if (m == 0) return 0;
+    if (!A || !B || !G) return set_err(BULKGCD_EINVAL, "null pointer with m > 0");
+    if (mode == BULKGCD_MODE_RSA) {
+        int rc = check_moduli(A, m, W);
+        if (!rc) rc = check_moduli(B, m, W);
+        if (rc) return rc;
+    }
+    int rc = device_check();
+    if (rc) return rc;
+    cudaStream_t st = cudaStreamPerThread;
+    size_t m_pad = pad32(m), rm = m * W * 4, cm = m_pad * W * 4;
+    DBuf dA, dB, dAc, dBc, dGc, dIt, dS;
+    CK(dA.alloc(rm, st));
+    CK(dB.alloc(rm, st));
+    CK(dAc.alloc(cm, st));
+    CK(dBc.alloc(cm, st));
+    CK(dGc.alloc(cm, st));
+    CK(dS.alloc(4 * sizeof(unsigned long long), st));
+    if (iters) CK(dIt.alloc(m * 4, st));
+    CK(cudaMemcpyAsync(dA.p, A, rm, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(dB.p, B, rm, cudaMemcpyHostToDevice, st));
+    if ((rc = bulkgcd_interleave(dA.as<uint32_t>(), dAc.as<uint32_t>(), m, m_pad, bits, 1, st))) return rc;
+    if ((rc = bulkgcd_interleave(dB.as<uint32_t>(), dBc.as<uint32_t>(), m, m_pad, bits, 1, st))) return rc;
+    if ((rc = bulkgcd_pairs_device(dAc.as<uint32_t>(), dBc.as<uint32_t>(), dGc.as<uint32_t>(), m, m_pad, bits, mode,
+                                   iters ? dIt.as<uint32_t>() : nullptr, dS.as<unsigned long long>(), 0, st)))
+        return rc;
+    // de-interleave into dA (reused as the row-major result buffer)
+    if ((rc = bulkgcd_interleave(dGc.as<uint32_t>(), dA.as<uint32_t>(), m, m_pad, bits, 0, st))) return rc;
+    CK(cudaMemcpyAsync(G, dA.p, rm, cudaMemcpyDeviceToHost, st));
+    if (iters) CK(cudaMemcpyAsync(iters, dIt.p, m * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    return 0;
+}
+
+int bulkgcd_pairs(const uint32_t *A, const uint32_t *B, size_t m, uint32_t bits, uint32_t *G) {
+    return bulkgcd_pairs_ex(A, B, m, bits, BULKGCD_MODE_EXACT, G, nullptr);
+}
+
+void bulkgcd_hits_free(bulkgcd_hits_t *h) {
+    if (!h) return;
+    free(h->ij);
+    free(h->gcd);
+    h->ij = nullptr;
+    h->gcd = nullptr;
+    h->count = 0;
+}
+
+int bulkgcd_all_pairs(const uint32_t *N, size_t n, uint32_t bits, bulkgcd_hits_t *out) {
+    int W = words_for(bits);
+    if (!out) return set_err(BULKGCD_EINVAL, "null hits_out");
+    memset(out, 0, sizeof *out);
+    out->bits = bits;
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048)", bits);
+    if (n > 0 && !N) return set_err(BULKGCD_EINVAL, "null moduli with n > 0");
+    if (n > 0xFFFFFFFFull) return set_err(BULKGCD_EINVAL, "n too large");
+    int rc = check_moduli(N, n, W);
+    if (rc) return rc;
+    if (n < 2) return 0;
+    if ((rc = device_check())) return rc;
+    cudaStream_t st = cudaStreamPerThread;
+    DBuf dN, dBlk, dC, dH;
+    CK(dN.alloc(n * W * 4, st));
+    CK(dBlk.alloc(bulkgcd_blocked_words(n, bits) * 4, st));
+    CK(dC.alloc(4 * sizeof(unsigned long long), st));
+    CK(cudaMemcpyAsync(dN.p, N, n * W * 4, cudaMemcpyHostToDevice, st));
+    if ((rc = bulkgcd_layout_blocked(dN.as<uint32_t>(), dBlk.as<uint32_t>(), n, bits, st))) return rc;
+    uint64_t cap = 1024;
+    uint64_t total = cohort_total(n);
+    unsigned long long count = 0;
+    for (int attempt = 0; attempt < 3; ++attempt) {
+        if (dH.p) {
+            cudaFreeAsync(dH.p, st);
+            dH.p = nullptr;
+        }
+        CK(dH.alloc(cap * (2 + W) * 4, st));
+        if ((rc = bulkgcd_all_pairs_band(dN.as<uint32_t>(), dBlk.as<uint32_t>(), n, bits, 0, total,
+                                         dH.as<uint32_t>(), cap, dC.as<unsigned long long>(), 0, st)))
+            return rc;
+        CK(cudaMemcpyAsync(&count, dC.p, sizeof count, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (count <= cap) break;
+        cap = count;  // overflow: rerun with room for every hit
+    }
+    if (count > cap) return set_err(BULKGCD_ECUDA, "hit buffer overflow persisted");
+    std::vector<uint32_t> rec(count * (2 + W));
+    if (count) CK(cudaMemcpyAsync(rec.data(), dH.p, rec.size() * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    std::vector<size_t> order(count);
+    std::iota(order.begin(), order.end(), 0);
+    std::sort(order.begin(), order.end(), [&](size_t a, size_t b) {
+        const uint32_t *ra = &rec[a * (2 + W)], *rb = &rec[b * (2 + W)];
+        return ra[0] != rb[0] ? ra[0] < rb[0] : ra[1] < rb[1];
+    });
+    if (count) {
+        out->ij = (uint32_t(*)[2])malloc(count * sizeof(uint32_t[2]));
+        out->gcd = (uint32_t *)malloc(count * W * sizeof(uint32_t));
+        if (!out->ij || !out->gcd) {
+            bulkgcd_hits_free(out);
+            return set_err(BULKGCD_ENOMEM, "host allocation of %llu hits failed", count);
+        }
+        for (size_t h = 0; h < count; ++h) {
+            const uint32_t *r = &rec[order[h] * (2 + W)];
+            out->ij[h][0] = r[0];
+            out->ij[h][1] = r[1];
+            memcpy(out->gcd + h * W, r + 2, W * 4);
+        }
+    }
+    out->count = count;
+    out->bits = bits;
+    return 0;
+}
+
+}  // extern "C"

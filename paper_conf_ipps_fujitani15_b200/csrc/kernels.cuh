@@ -1,0 +1,414 @@
+// kernels.cuh -- the bulk GCD kernels (sm_100a): layout transforms, the
+// independent-pairs kernel (bulkgcd_pairs) and the all-pairs kernel
+// (bulkgcd_all_pairs / bulkgcd_all_pairs_band).
+#pragma once
+#include <cstdint>
+
+#include "euclid.cuh"
+
+namespace bulkgcd {
+
+constexpr int THREADS = 128;  // 4 warps per CTA
+#ifndef MIN_BLOCKS
+#define MIN_BLOCKS 4  // CTAs per SM (4 -> <= 128 registers per thread)
+#endif
+
+// ------------------------------------------------------------------ layouts
+// Word-interleaved ("column-wise", PAPER.md L361 and Fig. 3) layouts: lane t of
+// a warp reads word k of its operand at consecutive addresses, so every limb
+// load is one coalesced 128-byte transaction.
+//   interleaved: X_cm[k * m_pad + i]
+//   blocked    : X_blk[(b * W + k) * 32 + t] for i = 32 b + t  (one cohort's 32
+//                operands are a contiguous W*128-byte block)
+
+// row-major [m][W] -> interleaved [W][m_pad] (to_cm) or back.
+__global__ void interleave_kernel(const uint32_t *__restrict__ in, uint32_t *__restrict__ out, uint64_t m,
+                                  uint64_t m_pad, int W, int to_cm) {
+    __shared__ uint32_t tile[32][33];
+    uint64_t i0 = (uint64_t)blockIdx.x * 32;
+    int k0 = blockIdx.y * 32;
+    int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
+    for (int r = ty; r < 32; r += 8) {
+        if (to_cm) {  // read row-major: row i0+r, word k0+tx
+            uint64_t i = i0 + r;
+            int k = k0 + tx;
+            tile[r][tx] = (i < m && k < W) ? in[i * W + k] : 0u;
+        } else {  // read interleaved: word k0+r, item i0+tx
+            uint64_t i = i0 + tx;
+            int k = k0 + r;
+            tile[tx][r] = (i < m_pad && k < W) ? in[(uint64_t)k * m_pad + i] : 0u;
+        }
+    }
+    __syncthreads();
+    for (int r = ty; r < 32; r += 8) {
+        if (to_cm) {  // write interleaved: word k0+r, item i0+tx
+            uint64_t i = i0 + tx;
+            int k = k0 + r;
+            if (i < m_pad && k < W) out[(uint64_t)k * m_pad + i] = tile[tx][r];
+        } else {  // write row-major
+            uint64_t i = i0 + r;
+            int k = k0 + tx;
+            if (i < m && k < W) out[i * W + k] = tile[r][tx];
+        }
+    }
+}
+
+// row-major [n][W] -> blocked [nb][W][32] (zero padded).
+__global__ void blocked_kernel(const uint32_t *__restrict__ in, uint32_t *__restrict__ out, uint64_t n, int W) {
+    __shared__ uint32_t tile[32][33];
+    uint64_t b = blockIdx.x;
+    int k0 = blockIdx.y * 32;
+    int tx = threadIdx.x, ty = threadIdx.y;
+    for (int r = ty; r < 32; r += 8) {
+        uint64_t i = b * 32 + r;
+        int k = k0 + tx;
+        tile[r][tx] = (i < n && k < W) ? in[i * W + k] : 0u;
+    }
+    __syncthreads();
+    for (int r = ty; r < 32; r += 8) {
+        int k = k0 + r;
+        if (k < W) out[(b * W + k) * 32 + tx] = tile[tx][r];
+    }
+}
+
+// ------------------------------------------------------------ lane helpers
+__device__ __forceinline__ uint64_t small_value(int l, uint64_t t) {
+    return l >= 2 ? t : (l == 1 ? (t >> 32) : 0ull);
+}
+
+__device__ __forceinline__ int bitlen_top(int l, uint64_t t) {
+    return l == 0 ? 0 : 32 * (l - 1) + (32 - __clz(hi32(t)));
+}
+
+// Order a lane's fresh operands so that A >= B, and compute lengths and tops.
+template <int W>
+__device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
+                                           uint64_t &tB) {
+    lA = scan_full<W>(A, tA) + 1;
+    lB = scan_full<W>(B, tB) + 1;
+    int c = lA != lB ? (lA < lB ? -1 : 1) : (tA != tB ? (tA < tB ? -1 : 1) : 0);
+    if (c == 0) {  // equal lengths and tops: full compare, most significant first
+#pragma unroll
+        for (int k = W - 1; k >= 0; --k)
+            if (c == 0 && A[k] != B[k]) c = A[k] < B[k] ? -1 : 1;
+    }
+    if (c < 0) {
+        swap_regs<W>(A, B);
+        int tl = lA; lA = lB; lB = tl;
+        uint64_t tt = tA; tA = tB; tB = tt;
+    }
+}
+
+// The per-cohort Euclid loop.  A >= B on entry (registers least-significant
+// first, s = 0).  cond(lX, tX, lY, tY) says whether a lane keeps iterating
+// (the do-while condition); sink(...) is called, warp-converged, whenever at
+// least one lane stops, with fin = "this lane stopped now" and X/Y its operands.
+template <int W, bool STATS, class Cond, class Sink>
+__device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
+                                            uint64_t &tB, bool live, Cond cond, Sink &sink, uint32_t &iters,
+                                            uint32_t &nslow) {
+    int s = 0;
+    for (;;) {
+        bool run = live && cond(lA, tA, lB, tB);
+        bool fin = live && !run;
+        if (__any_sync(FULL, fin)) sink(fin, A, B, lA, tA, lB, tB, s);
+        live = run;
+        if (!__any_sync(FULL, run)) break;
+        realign<W>(A, B, s, run ? lA : 0);
+        fast_iter<W, STATS>(A, B, lA, tA, lB, tB, s, run, iters, nslow);
+
+        run = live && cond(lB, tB, lA, tA);
+        fin = live && !run;
+        if (__any_sync(FULL, fin)) sink(fin, B, A, lB, tB, lA, tA, s);
+        live = run;
+        if (!__any_sync(FULL, run)) break;
+        realign<W>(A, B, s, run ? lB : 0);
+        fast_iter<W, STATS>(B, A, lB, tB, lA, tA, s, run, iters, nslow);
+    }
+}
+
+// RSA-mode loop condition (early-terminate, L243/L251/L255): continue while Y
+// has at least s/2 bits.
+struct RsaCond {
+    int half;
+    __device__ __forceinline__ bool operator()(int lX, uint64_t tX, int lY, uint64_t tY) const {
+        return bitlen_top(lY, tY) >= half;
+    }
+};
+
+// Exact-mode condition: continue while Y != 0 and X has >= 3 words (Case 1,
+// lX <= 2, finishes in the 64-bit tail).
+struct ExactCond {
+    __device__ __forceinline__ bool operator()(int lX, uint64_t tX, int lY, uint64_t tY) const {
+        return lY >= 1 && lX >= 3;
+    }
+};
+
+// -------------------------------------------------------------- generic I/O
+// Write g << k2 (g: n words in local memory) as W output words.
+template <int W>
+__device__ __noinline__ void write_shifted(uint32_t *out, uint64_t stride, const uint32_t *g, int n, int k2) {
+    int q = k2 >> 5, b = k2 & 31;
+    for (int w = 0; w < W; ++w) {
+        int src = w - q;
+        uint32_t lo = (src >= 0 && src < n) ? g[src] : 0u;
+        uint32_t lo1 = (src - 1 >= 0 && src - 1 < n) ? g[src - 1] : 0u;
+        uint32_t v = b ? ((lo << b) | (lo1 >> (32 - b))) : lo;
+        out[(uint64_t)w * stride] = v;
+    }
+}
+
+// Exact-mode normalisation: gcd(x, 0) = x; strip the common
+// power of two k2 = min(ctz a, ctz b) and all other trailing zeros.
+// Returns 1 if the result is already known (a zero operand).
+template <int W>
+__device__ __forceinline__ int normalize_exact(uint32_t (&A)[W], uint32_t (&B)[W], int &k2) {
+    uint32_t a[W], b[W];
+#pragma unroll
+    for (int k = 0; k < W; ++k) {
+        a[k] = A[k];
+        b[k] = B[k];
+    }
+    int za = 0, zb = 0;
+    while (za < W && a[za] == 0) ++za;
+    while (zb < W && b[zb] == 0) ++zb;
+    if (za == W || zb == W) {  // gcd(x, 0) = x: leave x | 0 in A
+#pragma unroll
+        for (int k = 0; k < W; ++k) A[k] = a[k] | b[k];
+        k2 = 0;
+        return 1;
+    }
+    int ca = 32 * za + ctz32(a[za]);
+    int cb = 32 * zb + ctz32(b[zb]);
+    k2 = ca < cb ? ca : cb;
+    n_rshift(a, W);
+    n_rshift(b, W);
+#pragma unroll
+    for (int k = 0; k < W; ++k) {
+        A[k] = a[k];
+        B[k] = b[k];
+    }
+    return 0;
+}
+
+// ------------------------------------------------------------ pairs kernel
+// G[i] = gcd(A[i], B[i]), i < m; operands and results word-interleaved.
+// EXACT: full gcd of any operands (L41 + Approximate Euclid to Y = 0).
+// RSA  : early-terminate; G = g if bitlen(g) >= bits/2 else 1.
+struct PairsArgs {
+    const uint32_t *A;
+    const uint32_t *B;
+    uint32_t *G;
+    uint64_t m, m_pad;
+    unsigned long long *work;  // cohort cursor, zeroed by the host
+    uint32_t *iters;           // optional per-pair iteration counts
+    unsigned long long *stats; // optional [sum iterations, slow steps]
+    int half;
+};
+
+template <int W>
+struct PairsSinkExact {
+    uint32_t *G;
+    uint64_t i, stride;
+    int k2;
+    bool tail;
+    uint64_t x64, y64;
+    __device__ __forceinline__ void operator()(bool fin, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX,
+                                               int lY, uint64_t tY, int s) {
+        if (!fin) return;
+        if (lY == 0) {  // Y = 0: g = X (may be long)
+            uint32_t g[W];
+#pragma unroll
+            for (int k = 0; k < W; ++k) g[k] = X[k];
+            write_shifted<W>(G + i, stride, g + s, W - s, k2);
+        } else {  // lX <= 2: Case 1 from here on, in 64-bit scalars
+            tail = true;
+            x64 = small_value(lX, tX);
+            y64 = small_value(lY, tY);
+        }
+    }
+};
+
+template <int W>
+struct PairsSinkRsa {
+    uint32_t *G;
+    uint64_t i, stride;
+    __device__ __forceinline__ void operator()(bool fin, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX,
+                                               int lY, uint64_t tY, int s) {
+        if (!fin) return;
+        if (lY == 0) {
+            uint32_t g[W];
+#pragma unroll
+            for (int k = 0; k < W; ++k) g[k] = X[k];
+            write_shifted<W>(G + i, stride, g + s, W - s, 0);
+        } else {
+            for (int w = 0; w < W; ++w) G[i + (uint64_t)w * stride] = w == 0 ? 1u : 0u;
+        }
+    }
+};
+
+template <int W, bool RSA, bool STATS>
+__global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a) {
+    const int lane = threadIdx.x & 31;
+    uint32_t iters = 0, nslow = 0;
+    for (;;) {
+        unsigned long long c = 0;
+        if (lane == 0) c = atomicAdd(a.work, 1ull);
+        c = __shfl_sync(FULL, c, 0);
+        uint64_t i = c * 32 + lane;
+        if (c * 32 >= a.m) break;
+        bool valid = i < a.m;
+        uint32_t A[W], B[W];
+#pragma unroll
+        for (int k = 0; k < W; ++k) {
+            A[k] = valid ? a.A[(uint64_t)k * a.m_pad + i] : 0u;
+            B[k] = valid ? a.B[(uint64_t)k * a.m_pad + i] : 0u;
+        }
+        uint32_t it0 = iters;
+        int lA, lB;
+        uint64_t tA, tB;
+        if (RSA) {
+            bool live = valid;
+            setup_pair<W>(A, B, lA, tA, lB, tB);
+            PairsSinkRsa<W> sink{a.G, i, a.m_pad};
+            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow);
+        } else {
+            int k2 = 0;
+            bool known = false;
+            if (valid) known = normalize_exact<W>(A, B, k2) != 0;
+            if (valid && known) {
+#pragma unroll
+                for (int k = 0; k < W; ++k) a.G[i + (uint64_t)k * a.m_pad] = A[k];
+            }
+            bool live = valid && !known;
+            if (!live) {
+#pragma unroll
+                for (int k = 0; k < W; ++k) A[k] = B[k] = 0;
+            }
+            setup_pair<W>(A, B, lA, tA, lB, tB);
+            PairsSinkExact<W> sink{a.G, i, a.m_pad, k2, false, 0, 0};
+            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, iters, nslow);
+            // 64-bit tail: Case 1 of approx (lX <= 2): alpha = X div Y, exactly (L127).
+            if (sink.tail) {
+                uint64_t x = sink.x64, y = sink.y64;
+                while (y != 0) {
+                    uint64_t q = x / y;
+                    if ((q & 1) == 0) q -= 1;
+                    x = x - y * q;
+                    if (x) x >>= __ffsll((long long)x) - 1;
+                    if (x < y) { uint64_t t = x; x = y; y = t; }
+                    if (STATS) ++iters;
+                }
+                uint32_t g[2] = {lo32(x), hi32(x)};
+                write_shifted<W>(a.G + i, a.m_pad, g, 2, sink.k2);
+            }
+        }
+        if (a.iters && valid) a.iters[i] = iters - it0;
+    }
+    if (STATS && a.stats) {
+        atomicAdd(&a.stats[0], (unsigned long long)iters);
+        atomicAdd(&a.stats[1], (unsigned long long)nslow);
+    }
+}
+
+// --------------------------------------------------------- all-pairs kernel
+// Work unit = cohort = (row block b of 32 consecutive moduli, column j), j >
+// 32 b; lane t takes the pair (32 b + t, j) if 32 b + t < j.  Cohorts are
+// numbered row block by row block: P(b) = b (n - 1) - 16 b (b - 1) cohorts
+// precede row block b.  Every pair i < j is in exactly one cohort, and a
+// contiguous range of cohort ids is a balanced share of the triangle (the
+// multi-GPU band partition).
+__host__ __device__ __forceinline__ uint64_t cohorts_before(uint64_t b, uint64_t n) {
+    return b * (n - 1) - 16 * b * (b - 1);
+}
+
+__host__ __device__ __forceinline__ uint64_t cohort_total(uint64_t n) {
+    if (n < 2) return 0;
+    uint64_t nb = (n + 31) / 32;
+    return cohorts_before(nb, n);
+}
+
+struct AllPairsArgs {
+    const uint32_t *N_blk;  // blocked [nb][W][32]
+    const uint32_t *N_rm;   // row-major [n][W]
+    uint64_t n;
+    uint64_t c_begin, c_end;
+    unsigned long long *work;      // cursor, zeroed by the host
+    uint32_t *hits;                // hit records [i, j, g[W]]
+    uint64_t hit_cap;
+    unsigned long long *hit_count;
+    unsigned long long *stats;     // optional [sum iterations, slow steps]
+    int half;
+};
+
+template <int W>
+struct HitSink {
+    uint32_t *hits;
+    uint64_t cap;
+    unsigned long long *count;
+    uint32_t i, j;
+    __device__ __forceinline__ void operator()(bool fin, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX,
+                                               int lY, uint64_t tY, int s) {
+        // Compacting hit writer: warp ballot + one atomic per warp (north_star (4)).
+        bool hit = fin && lY == 0;
+        unsigned mask = __ballot_sync(FULL, hit);
+        if (mask == 0) return;
+        const int lane = threadIdx.x & 31;
+        unsigned long long base = 0;
+        if (lane == __ffs(mask) - 1) base = atomicAdd(count, (unsigned long long)__popc(mask));
+        base = __shfl_sync(FULL, base, __ffs(mask) - 1);
+        if (!hit) return;
+        uint64_t slot = base + __popc(mask & ((1u << lane) - 1));
+        if (slot >= cap) return;  // counted, not written: the host retries with more room
+        uint32_t *rec = hits + slot * (2 + W);
+        rec[0] = i;
+        rec[1] = j;
+#pragma unroll
+        for (int k = 0; k < W; ++k) {
+            if (k >= s) rec[2 + k - s] = X[k];
+            if (k >= W - s) rec[2 + k] = 0u;
+        }
+    }
+};
+
+template <int W, bool STATS>
+__global__ void __launch_bounds__(THREADS, MIN_BLOCKS) allpairs_kernel(AllPairsArgs a) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t nb = (a.n + 31) / 32;
+    uint32_t iters = 0, nslow = 0;
+    for (;;) {
+        unsigned long long c = 0;
+        if (lane == 0) c = atomicAdd(a.work, 1ull);
+        c = __shfl_sync(FULL, c, 0) + a.c_begin;
+        if (c >= a.c_end) break;
+        // cohort id -> (row block b, column j): largest b with P(b) <= c
+        uint64_t lo = 0, hi = nb;  // P(lo) <= c < P(hi)
+        while (hi - lo > 1) {
+            uint64_t mid = (lo + hi) / 2;
+            if (cohorts_before(mid, a.n) <= c) lo = mid; else hi = mid;
+        }
+        uint64_t b = lo;
+        uint64_t j = 32 * b + 1 + (c - cohorts_before(b, a.n));
+        uint64_t i = 32 * b + lane;
+        bool live = i < j;
+        uint32_t A[W], B[W];
+        const uint32_t *rowp = a.N_blk + b * W * 32 + lane;
+        const uint32_t *colp = a.N_rm + j * W;
+#pragma unroll
+        for (int k = 0; k < W; ++k) {
+            A[k] = rowp[k * 32];
+            B[k] = colp[k];
+        }
+        int lA, lB;
+        uint64_t tA, tB;
+        setup_pair<W>(A, B, lA, tA, lB, tB);
+        HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
+        euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow);
+    }
+    if (STATS && a.stats) {
+        atomicAdd(&a.stats[0], (unsigned long long)iters);
+        atomicAdd(&a.stats[1], (unsigned long long)nslow);
+    }
+}
+
+}  // namespace bulkgcd

@@ -1,0 +1,195 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bit-exact on every gcd value and on the exact hit set; per-pair iteration
+counts against the paper-algorithm model (the kernels implement the same
+exact-floor approx(), so the counts must agree pair by pair).
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from oracle import approx_model as am
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def bg():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_fujitani15_b200 as bg
+    bg.bulkgcd_device_check()
+    return bg
+
+
+# ------------------------------------------------------------------ pairs
+@pytest.mark.parametrize("bits,count", [(512, 3000), (1024, 5000), (2048, 1500)])
+def test_pairs_exact_mixed(bg, bits, count):
+    """Exact mode on every rare-path category (even, zero, beta > 0, r >= 32,
+    Cases 1-4, duplicates, common factors), a ragged count (not a multiple of 32)."""
+    W = bits // 32
+    A, B = synth.mixed_pairs(count, bits, seed=bits + 1)
+    Ah, Bh = synth.from_ints(A, W), synth.from_ints(B, W)
+    G = bg.bulkgcd_pairs(Ah, Bh, bits)
+    want = oracle.gcd_batch(Ah, Bh)
+    bad = np.nonzero(~np.all(G == want, axis=1))[0]
+    assert bad.size == 0, [(int(k), A[k], B[k]) for k in bad[:3]]
+
+
+def test_pairs_exact_iteration_parity(bg):
+    bits, W = 1024, 32
+    A, B = synth.mixed_pairs(1100, bits, seed=77)
+    ms = synth.moduli(400, bits, seed=78)
+    N = synth.ints(ms.N)
+    A += N[:200]
+    B += N[200:]
+    Ah, Bh = synth.from_ints(A, W), synth.from_ints(B, W)
+    G, it = bg.bulkgcd_pairs_ex(Ah, Bh, bits, bg.MODE_EXACT, want_iters=True)
+    for k, (a, b) in enumerate(zip(A, B)):
+        t = am.gcd_exact(a, b)
+        assert synth.to_int(G[k]) == t.gcd == math.gcd(a, b)
+        assert int(it[k]) == t.iterations, (k, a, b, int(it[k]), t.iterations)
+
+
+@pytest.mark.parametrize("bits", [512, 1024, 2048])
+def test_pairs_rsa_mode(bg, bits):
+    W = bits // 32
+    ms = synth.moduli(801, bits, seed=900 + bits, n_planted_pairs=20, n_duplicates=3)
+    N = synth.ints(ms.N)
+    rng = np.random.default_rng(bits)
+    ii = list(range(800)) + [a for a, b, _ in ms.truth]
+    jj = [int(x) for x in rng.integers(0, 801, size=800)] + [b for a, b, _ in ms.truth]
+    A = [N[i] for i in ii]
+    B = [N[j] for j in jj]
+    Ah, Bh = synth.from_ints(A, W), synth.from_ints(B, W)
+    G, it = bg.bulkgcd_pairs_ex(Ah, Bh, bits, bg.MODE_RSA, want_iters=True)
+    Gx = oracle.gcd_batch(Ah, Bh)
+    hit = oracle.rsa_hit(oracle.bitlen_rows(Gx), bits)
+    for k in range(len(A)):
+        want = synth.to_int(Gx[k]) if hit[k] else 1
+        assert synth.to_int(G[k]) == want, k
+        t = am.gcd_rsa(A[k], B[k], bits)
+        assert t.gcd == want
+        assert int(it[k]) == t.iterations, (k, int(it[k]), t.iterations)
+
+
+def test_pairs_edge_cases(bg):
+    W = 32
+    assert bg.bulkgcd_pairs(np.zeros((0, W), np.uint32), np.zeros((0, W), np.uint32), 1024).shape == (0, W)
+    top = (1 << 1024) - 1
+    A = [0, 0, 5, top, top, top - 2, 1 << 1023, 1, 3 ** 600, (1 << 1023) + 1]
+    B = [0, 7, 0, top, top - 2, top, 1 << 1000, top, 3 ** 500, (1 << 1023) + 1]
+    Ah, Bh = synth.from_ints(A, W), synth.from_ints(B, W)
+    G = bg.bulkgcd_pairs(Ah, Bh, 1024)
+    assert [synth.to_int(g) for g in G] == [math.gcd(a, b) for a, b in zip(A, B)]
+
+
+def test_pairs_errors(bg):
+    W = 32
+    Z = np.zeros((1, W), np.uint32)
+    with pytest.raises(bg.BulkGcdError) as e:
+        bg.bulkgcd_pairs_ex(Z, Z, 1024, bg.MODE_RSA)  # RSA mode needs odd moduli > 1
+    assert e.value.code == bg.EINVAL
+    with pytest.raises(bg.BulkGcdError) as e:
+        bg.bulkgcd_pairs(np.zeros((1, 3), np.uint32), np.zeros((1, 3), np.uint32), 96)
+    assert e.value.code == bg.EINVAL
+
+
+# -------------------------------------------------------------- all pairs
+def test_all_pairs_config1(bg, cfg1):
+    hits = bg.bulkgcd_all_pairs(cfg1.N, 1024).as_list()
+    assert hits == oracle.all_pairs_hits(cfg1.N, 1024) == cfg1.truth
+
+
+@pytest.mark.parametrize("n,bits", [(2, 1024), (33, 1024), (95, 512), (70, 2048), (161, 1024)])
+def test_all_pairs_exhaustive_small(bg, n, bits):
+    """Every pair checked by the oracle; ragged n; cliques and duplicates."""
+    ms = synth.moduli(n, bits, seed=n * 7 + bits, n_planted_pairs=min(3, n // 2),
+                      cliques=(4,) if n >= 33 else (), n_duplicates=2 if n >= 33 else 0)
+    hits = bg.bulkgcd_all_pairs(ms.N, bits).as_list()
+    assert hits == oracle.all_pairs_hits(ms.N, bits) == ms.truth
+
+
+def test_all_pairs_errors(bg, cfg1):
+    N = cfg1.N.copy()
+    N[5, 0] &= ~np.uint32(1)
+    with pytest.raises(bg.BulkGcdError) as e:
+        bg.bulkgcd_all_pairs(N, 1024)
+    assert e.value.code == bg.EINVAL
+    one = cfg1.N[:3].copy()
+    one[1] = 0
+    one[1, 0] = 1
+    with pytest.raises(bg.BulkGcdError):
+        bg.bulkgcd_all_pairs(one, 1024)
+    assert bg.bulkgcd_all_pairs(cfg1.N[:1], 1024).ij.shape == (0, 2)
+
+
+def _band_run(bg, ms, bits, c0, c1, cap):
+    W = bits // 32
+    dev = torch.device("cuda")
+    dN = torch.from_numpy(ms.N.view(np.int32)).to(dev)
+    dB = torch.empty(bg.bulkgcd_blocked_words(ms.m, bits), dtype=torch.int32, device=dev)
+    bg.bulkgcd_layout_blocked(dN, dB, ms.m, bits)
+    dH = torch.zeros(max(cap, 1) * (2 + W), dtype=torch.int32, device=dev)
+    dC = torch.zeros(4, dtype=torch.int64, device=dev)
+    bg.bulkgcd_all_pairs_band(dN, dB, ms.m, bits, c0, c1, dH, cap, dC, bg.FLAG_STATS)
+    torch.cuda.synchronize()
+    count = int(dC[0].item())
+    rec = dH.cpu().numpy().view(np.uint32).reshape(-1, 2 + W)[:min(count, cap)]
+    out = sorted((int(r[0]), int(r[1]), synth.to_int(r[2:])) for r in rec)
+    return count, out, dC.cpu().numpy()
+
+
+def test_band_partition_and_overflow(bg):
+    ms = synth.moduli(300, 1024, seed=31, n_planted_pairs=6, cliques=(3,))
+    total = bg.bulkgcd_cohort_count(ms.m)
+    full = []
+    for parts in (1, 2, 3, 8):
+        cuts = [total * p // parts for p in range(parts + 1)]
+        got = []
+        for p in range(parts):
+            c, out, _ = _band_run(bg, ms, 1024, cuts[p], cuts[p + 1], 64)
+            assert c == len(out)
+            got += out
+        got.sort()
+        if parts == 1:
+            full = got
+        assert got == full == ms.truth
+    # fault injection: a hit buffer too small for the band is counted, not overrun
+    c, out, _ = _band_run(bg, ms, 1024, 0, total, 2)
+    assert c == len(ms.truth) and len(out) == 2 and set(out) <= set(ms.truth)
+
+
+def test_all_pairs_stats_counters(bg, cfg1):
+    total = bg.bulkgcd_cohort_count(cfg1.m)
+    _, _, ctr = _band_run(bg, cfg1, 1024, 0, total, 16)
+    N = synth.ints(cfg1.N)
+    want = sum(am.gcd_rsa(N[i], N[j], 1024).iterations for i in range(64) for j in range(i + 1, 64))
+    assert int(ctr[2]) == want
+
+
+@pytest.mark.slow
+def test_all_pairs_config3_full(bg):
+    """BASELINE configs[2] at full size, in the launch configuration bench.py times:
+    the exact hit set against construction ground truth, and a seeded sample of
+    pairs whose oracle gcd must then be < 2^(bits/2)."""
+    ms = synth.config_moduli(3)
+    hits = bg.bulkgcd_all_pairs(ms.N, 1024).as_list()
+    assert hits == ms.truth
+    rng = np.random.default_rng(3)
+    ii = rng.integers(0, ms.m, size=20000)
+    jj = rng.integers(0, ms.m, size=20000)
+    keep = ii < jj
+    ii, jj = ii[keep], jj[keep]
+    G = oracle.gcd_index_pairs(ms.N, ii, jj)
+    hit = oracle.rsa_hit(oracle.bitlen_rows(G), 1024)
+    truth = {(a, b) for a, b, _ in ms.truth}
+    for k in range(ii.size):
+        assert bool(hit[k]) == ((int(ii[k]), int(jj[k])) in truth)
+    # planted pairs through the oracle, gcd by gcd
+    for a, b, g in ms.truth:
+        assert oracle.gcd(synth.to_int(ms.N[a]), synth.to_int(ms.N[b])) == g
