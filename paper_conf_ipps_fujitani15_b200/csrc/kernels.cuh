@@ -10,7 +10,7 @@ namespace bulkgcd {
 
 constexpr int THREADS = 128;  // 4 warps per CTA
 #ifndef MIN_BLOCKS
-#define MIN_BLOCKS 4  // CTAs per SM (4 -> <= 128 registers per thread)
+#define MIN_BLOCKS 3  // CTAs per SM (3 -> <= 168 registers per thread, no spills)
 #endif
 
 // ------------------------------------------------------------------ layouts
@@ -100,30 +100,90 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 }
 
 // The per-cohort Euclid loop.  A >= B on entry (registers least-significant
-// first, s = 0).  cond(lX, tX, lY, tY) says whether a lane keeps iterating
-// (the do-while condition); sink(...) is called, warp-converged, whenever at
-// least one lane stops, with fin = "this lane stopped now" and X/Y its operands.
+// first, s = 0).  cond(lX, tX, lY, tY) is the do-while condition of a lane.
+//
+// Structure: a hot loop (two iterations per trip with exchanged roles) that
+// touches the operand registers only through the fused pass, and a cold
+// section that handles everything rare -- fix-ups (no swap, slow path),
+// finished lanes whose result needs the operand registers (sink), and the
+// realign when the warp length L dropped.  Keeping every conditional write of
+// the register arrays out of the hot loop stops ptxas from materialising
+// whole-array copies at merge points.
+//
+// Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
+// and returns true if a finished lane needs cold(...) (warp-converged, with
+// the operand registers); scalar-only finishes are handled by quick itself.
 template <int W, bool STATS, class Cond, class Sink>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, uint32_t &iters,
                                             uint32_t &nslow) {
     int s = 0;
-    for (;;) {
-        bool run = live && cond(lA, tA, lB, tB);
-        bool fin = live && !run;
-        if (__any_sync(FULL, fin)) sink(fin, A, B, lA, tA, lB, tB, s);
-        live = run;
-        if (!__any_sync(FULL, run)) break;
-        realign<W>(A, B, s, run ? lA : 0);
-        fast_iter<W, STATS>(A, B, lA, tA, lB, tB, s, run, iters, nslow);
+    int fix = 0;     // pending fix-up of the last iteration (hot_iter's code)
+    int resume = 0;  // roles of the next iteration: 0 -> (X, Y) = (A, B), 1 -> (B, A)
 
-        run = live && cond(lB, tB, lA, tA);
-        fin = live && !run;
-        if (__any_sync(FULL, fin)) sink(fin, B, A, lB, tB, lA, tA, s);
+    // Cold section for the next roles (X, Y); the last iteration ran on (Y, X).
+    auto cold = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
+        if (__any_sync(FULL, fix != 0)) {
+            if (STATS && fix >= 2) ++nslow;
+            apply_fix<W>(fix, Y, X, lY, tY, lX, tX, s);
+            fix = 0;
+        }
+        bool run = live && cond(lX, tX, lY, tY);
+        bool fin = live && !run;
+        if (__any_sync(FULL, fin)) {
+            bool need = sink.quick(fin, lX, tX, lY, tY);
+            if (__any_sync(FULL, need)) sink.cold(need, X, Y, lX, tX, lY, tY, s);
+        }
         live = run;
-        if (!__any_sync(FULL, run)) break;
-        realign<W>(A, B, s, run ? lB : 0);
-        fast_iter<W, STATS>(B, A, lB, tB, lA, tA, s, run, iters, nslow);
+        if (!__any_sync(FULL, run)) return false;
+        int L = __reduce_max_sync(FULL, (unsigned)(run ? lX : 0));
+        while (W - s > L) {
+            shift_up_1<W>(A);
+            shift_up_1<W>(B);
+            ++s;
+        }
+        return true;
+    };
+    // One hot iteration on roles (X, Y).  0: continue; 1: go cold before the
+    // iteration (same roles); 2: iteration done, fix-ups pending (roles flip).
+    auto hot = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> int {
+        bool run = live && cond(lX, tX, lY, tY);
+        bool fin = live && !run;
+        bool need = sink.quick(fin, lX, tX, lY, tY);
+        // Go cold if a finished lane needs its registers, or if no running lane
+        // reaches the top register any more (the warp length L dropped: realign;
+        // this also covers "no lane running").  lX <= W - s always holds.
+        bool top = run && lX == W - s;
+        if (__any_sync(FULL, need) || !__any_sync(FULL, top)) return 1;
+        live = run;
+        fix = hot_iter<W>(X, Y, lX, tX, lY, tY, s, run);
+        if (STATS && run) ++iters;
+        return __any_sync(FULL, fix != 0) ? 2 : 0;
+    };
+
+    for (;;) {
+        bool more = resume == 0 ? cold(A, B, lA, tA, lB, tB) : cold(B, A, lB, tB, lA, tA);
+        if (!more) return;
+        int rc;
+        if (resume == 1) {
+            rc = hot(B, A, lB, tB, lA, tA);
+            if (rc) {
+                resume = rc == 2 ? 0 : 1;
+                continue;
+            }
+        }
+        for (;;) {
+            rc = hot(A, B, lA, tA, lB, tB);
+            if (rc) {
+                resume = rc == 2 ? 1 : 0;
+                break;
+            }
+            rc = hot(B, A, lB, tB, lA, tA);
+            if (rc) {
+                resume = rc == 2 ? 0 : 1;
+                break;
+            }
+        }
     }
 }
 
@@ -132,7 +192,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
 struct RsaCond {
     int half;
     __device__ __forceinline__ bool operator()(int lX, uint64_t tX, int lY, uint64_t tY) const {
-        return bitlen_top(lY, tY) >= half;
+        return 32 * lY - (int)__clz(hi32(tY)) >= half;  // bitlen(Y); lY = 0 gives -32
     }
 };
 
@@ -213,19 +273,23 @@ struct PairsSinkExact {
     int k2;
     bool tail;
     uint64_t x64, y64;
-    __device__ __forceinline__ void operator()(bool fin, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX,
-                                               int lY, uint64_t tY, int s) {
-        if (!fin) return;
-        if (lY == 0) {  // Y = 0: g = X (may be long)
-            uint32_t g[W];
-#pragma unroll
-            for (int k = 0; k < W; ++k) g[k] = X[k];
-            write_shifted<W>(G + i, stride, g + s, W - s, k2);
-        } else {  // lX <= 2: Case 1 from here on, in 64-bit scalars
+    // lX <= 2 (Y != 0): Case 1 from here on, in 64-bit scalars (no registers needed)
+    __device__ __forceinline__ bool quick(bool fin, int lX, uint64_t tX, int lY, uint64_t tY) {
+        if (fin && lY != 0) {
             tail = true;
             x64 = small_value(lX, tX);
             y64 = small_value(lY, tY);
         }
+        return fin && lY == 0;
+    }
+    // Y = 0: g = X (possibly long), written with the common power of two restored
+    __device__ __forceinline__ void cold(bool need, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX, int lY,
+                                         uint64_t tY, int s) {
+        if (!need) return;
+        uint32_t g[W];
+#pragma unroll
+        for (int k = 0; k < W; ++k) g[k] = X[k];
+        write_shifted<W>(G + i, stride, g + s, W - s, k2);
     }
 };
 
@@ -233,9 +297,10 @@ template <int W>
 struct PairsSinkRsa {
     uint32_t *G;
     uint64_t i, stride;
-    __device__ __forceinline__ void operator()(bool fin, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX,
-                                               int lY, uint64_t tY, int s) {
-        if (!fin) return;
+    __device__ __forceinline__ bool quick(bool fin, int, uint64_t, int, uint64_t) { return fin; }
+    __device__ __forceinline__ void cold(bool need, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX, int lY,
+                                         uint64_t tY, int s) {
+        if (!need) return;
         if (lY == 0) {
             uint32_t g[W];
 #pragma unroll
@@ -347,16 +412,17 @@ struct HitSink {
     uint64_t cap;
     unsigned long long *count;
     uint32_t i, j;
-    __device__ __forceinline__ void operator()(bool fin, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX,
-                                               int lY, uint64_t tY, int s) {
-        // Compacting hit writer: warp ballot + one atomic per warp (north_star (4)).
-        bool hit = fin && lY == 0;
+    // a lane that stops with Y != 0 is coprime-mode ("return 1", L243/L251): nothing to report
+    __device__ __forceinline__ bool quick(bool fin, int, uint64_t, int lY, uint64_t) { return fin && lY == 0; }
+    // Compacting hit writer: warp ballot + one atomic per warp (north_star (4)).
+    __device__ __forceinline__ void cold(bool hit, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX, int lY,
+                                         uint64_t tY, int s) {
         unsigned mask = __ballot_sync(FULL, hit);
-        if (mask == 0) return;
         const int lane = threadIdx.x & 31;
+        const int leader = __ffs(mask) - 1;
         unsigned long long base = 0;
-        if (lane == __ffs(mask) - 1) base = atomicAdd(count, (unsigned long long)__popc(mask));
-        base = __shfl_sync(FULL, base, __ffs(mask) - 1);
+        if (lane == leader) base = atomicAdd(count, (unsigned long long)__popc(mask));
+        base = __shfl_sync(FULL, base, leader);
         if (!hit) return;
         uint64_t slot = base + __popc(mask & ((1u << lane) - 1));
         if (slot >= cap) return;  // counted, not written: the host retries with more room
