@@ -1,0 +1,375 @@
+#!/usr/bin/env python3
+"""bench.py -- all-pairs 1024-bit GCD throughput of libbulkgcd on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Workload (BASELINE.json metric "1024-bit GCDs/sec (all-pairs)", configs[2]):
+all 134,209,536 pairs (i < j) of 16,384 synthetic 1024-bit RSA moduli with 8
+planted shared primes (synth.config_moduli(3), seed 2018) -- the paper's
+Table V workload size.  One step = one full pass of the hot
+path: blocked layout of the resident moduli (H1), the all-pairs band kernel
+(H2-H9) and, for N > 1, the NCCL all-gather of the hit lists; N GPUs split the
+cohort range into balanced row bands (strong scaling: total work fixed).
+
+value   : device-timed (CUDA events, sum over the K steps, max over ranks),
+          moduli resident in HBM; L2 flushed (256 MiB write) before each step.
+e2e     : the same metric through the public API with HOST buffers: N = 1:
+          bulkgcd_all_pairs() (C ABI: H2D, kernels, D2H, sort); N > 1:
+          dist.all_pairs_distributed() per rank.  Host-timed per call.
+roofline: the all-pairs kernel, integer-issue bound ("alu"): algorithmic
+          lane-ops per launch (4 per limb-step + 16 per
+          iteration, counted exactly by the kernel's stats pass on the same
+          input) over its CUDA-event duration, against 148 SMs x 128 lanes x
+          the max SM clock of MEASURED_PEAKS.json.
+cpu_baseline (rank 0, N = 1): the C oracle (Original Euclid, oracle/) on a
+          bounded seeded sample of the same pairs, all host cores.
+--impl reference: the oracle as it stands is the reference arm (no reference
+          implementation exists; /root/reference is a paper).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PAPER_GCD_PER_S = 1.0 / 0.346e-6  # GTX 780 Ti, 1024-bit early-terminate, 16K all pairs
+METRIC = "1024-bit GCDs/sec (all-pairs)"
+UNIT = "GCD/s"
+OPS_PER_LIMB, OPS_PER_ITER = 4, 16  # SURVEY.md §8(d) M2; DESIGN.md §Roofline
+
+
+def _env_rank():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except OSError:
+        return {"sm_max_mhz": 1965.0}, "fallback"
+
+
+def _traffic():
+    """dram bytes per launch of the all-pairs kernel from the committed ncu summary."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as f:
+            s = json.load(f)
+        return s.get("allpairs_dram_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML while the timed region runs."""
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:  # no NVML: report what we have
+            self.nv = None
+
+    def _run(self):
+        nv = self.nv
+        names = {
+            "hw_slowdown": getattr(nv, "nvmlClocksThrottleReasonHwSlowdown", 0x8),
+            "sw_thermal_slowdown": getattr(nv, "nvmlClocksThrottleReasonSwThermalSlowdown", 0x20),
+            "hw_thermal_slowdown": getattr(nv, "nvmlClocksThrottleReasonHwThermalSlowdown", 0x40),
+            "sw_power_cap": getattr(nv, "nvmlClocksThrottleReasonSwPowerCap", 0x4),
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                for k, bit in names.items():
+                    if r & bit:
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            self._stop.wait(0.05)
+
+    def __enter__(self):
+        if self.nv is not None:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv is not None:
+            self.t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def cpu_baseline(ms, target_s: float = 12.0, seed: int = 7):
+    """The oracle (oracle/gcd_oracle.c, as it stands) on a bounded sample of the
+    workload's pairs, all host cores.  Returns the cpu_baseline object."""
+    import oracle
+    cores = os.cpu_count() or 1
+    rng = np.random.default_rng(seed)
+
+    def sample(k):
+        i = rng.integers(0, ms.m, size=2 * k)
+        j = rng.integers(0, ms.m, size=2 * k)
+        keep = i < j
+        return i[keep][:k], j[keep][:k]
+
+    i, j = sample(1 << 14)  # calibration
+    t0 = time.perf_counter()
+    oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
+    rate = i.size / (time.perf_counter() - t0)
+    k = int(min(1 << 23, max(1 << 16, rate * target_s)))
+    i, j = sample(k)
+    t0 = time.perf_counter()
+    oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
+    dt = time.perf_counter() - t0
+    return {"value": i.size / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{i.size} seeded random (i<j) pairs of the {ms.m}-moduli workload, exact classical Euclid "
+                      f"(Knuth D), {dt:.1f}s on {cores} threads"}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as the reference arm (rank 0 only)."""
+    rank, world, _ = _env_rank()
+    if rank != 0:
+        return
+    import synth
+    import oracle
+    ms = synth.config_moduli(3)
+    cores = os.cpu_count() or 1
+    per_step = 1 << 18
+    rng = np.random.default_rng(11)
+
+    def step():
+        i = rng.integers(0, ms.m, size=2 * per_step)
+        j = rng.integers(0, ms.m, size=2 * per_step)
+        keep = i < j
+        i, j = i[keep][:per_step], j[keep][:per_step]
+        t0 = time.perf_counter()
+        G = oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
+        dt = time.perf_counter() - t0
+        oracle.rsa_hit(oracle.bitlen_rows(G), 1024)
+        return i.size, dt
+
+    for _ in range(args.warmup):
+        step()
+    n_tot, t_tot = 0, 0.0
+    for _ in range(args.steps):
+        n, dt = step()
+        n_tot += n
+        t_tot += dt
+    v = n_tot / t_tot
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": t_tot / args.steps * 1e3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": v / PAPER_GCD_PER_S, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": "cfg3: all-pairs 1024-bit RSA moduli, n=16384 (134,209,536 pairs), 8 planted",
+                   "per_step_sample_pairs": per_step, "mode": "rsa-early-terminate (oracle: exact gcd + O3 map)"},
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": f"{per_step} seeded random (i<j) pairs per step, exact classical Euclid"},
+        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    if args.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    import paper_conf_ipps_fujitani15_b200 as bg
+    from paper_conf_ipps_fujitani15_b200 import dist as bgd
+
+    rank, world, local = _env_rank()
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world} (launch N>1 with torchrun)")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    bg.bulkgcd_device_check()
+
+    # ---- inputs: rank 0 generates the seeded moduli, NCCL broadcast to the others
+    bits = 1024
+    W = bits // 32
+    if rank == 0:
+        ms = synth.config_moduli(3)
+        N = ms.N
+        truth = ms.truth
+    else:
+        N = np.zeros((16384, W), np.uint32)
+        truth = None
+    if world > 1:
+        t = torch.from_numpy(N.view(np.int32)).to(dev)
+        dist.broadcast(t, 0)
+        N = t.cpu().numpy().view(np.uint32)
+    n = N.shape[0]
+    pairs = n * (n - 1) // 2
+
+    runner = bgd.AllPairsBand(N, bits, rank, world, device=dev)
+    runner.upload(non_blocking=False)
+    flush = torch.empty(64 << 20, dtype=torch.int32, device=dev)  # 256 MiB > 126 MB L2
+    cap = runner.cap
+    gbuf = torch.empty(world * cap * (2 + W), dtype=torch.int32, device=dev)
+    gcnt = torch.empty(world, dtype=torch.int64, device=dev)
+
+    def step():
+        runner.layout()
+        k0.record()
+        runner.search()
+        k1.record()
+        if world > 1:
+            # the exchange step: NCCL all-gather of the hit counts and fixed-capacity hit buffers
+            dist.all_gather_into_tensor(gcnt, runner.d_ctr[:1])
+            dist.all_gather_into_tensor(gbuf, runner.d_hits)
+
+    # ---- algorithmic work of one launch (stats pass, untimed)
+    runner.layout()
+    runner.search(bg.FLAG_STATS)
+    torch.cuda.synchronize()
+    ctr = runner.d_ctr.cpu().numpy().astype(np.int64)
+    iters, limbs = int(ctr[2]), int(ctr[4])
+    if world > 1:
+        tt = torch.tensor([iters, limbs], dtype=torch.int64, device=dev)
+        dist.all_reduce(tt)
+        iters, limbs = int(tt[0]), int(tt[1])
+    ops_alg = OPS_PER_LIMB * limbs + OPS_PER_ITER * iters  # whole job, per step
+
+    k0 = torch.cuda.Event(enable_timing=True)
+    k1 = torch.cuda.Event(enable_timing=True)
+    for _ in range(args.warmup):
+        flush.fill_(1)
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    step_ms, kern_ms = [], []
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t_wall = time.perf_counter()
+        for _ in range(args.steps):
+            flush.fill_(2)
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record()
+            step()
+            e1.record()
+            e1.synchronize()
+            step_ms.append(e0.elapsed_time(e1))
+            kern_ms.append(k0.elapsed_time(k1))
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t_wall = time.perf_counter() - t_wall
+
+    # correctness of the timed steps' output (outside the timed region)
+    local_hits = runner.local_hits()
+    if world > 1:
+        allrec = bgd.gather_hits(local_hits)
+    else:
+        allrec = local_hits
+    found = bgd.records_to_hits(allrec.cpu().numpy(), bits).as_list()
+    ok = (found == truth) if rank == 0 else True
+
+    tot_ms = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot_ms, op=dist.ReduceOp.MAX)
+    step_total_ms, kern_total_ms = float(tot_ms[0]), float(tot_ms[1])
+
+    # ---- end to end through the public API with host buffers
+    e2e_ms = []
+    Nh = np.ascontiguousarray(N)
+    d2h = 0
+    for _ in range(args.e2e_steps):
+        flush.fill_(3)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        if world == 1:
+            h = bg.bulkgcd_all_pairs(Nh, bits)
+        else:
+            h = bgd.all_pairs_distributed(Nh, bits)
+        dt = time.perf_counter() - t0
+        d2h = 8 + h.ij.shape[0] * (2 + W) * 4
+        e2e_ms.append(dt * 1e3)
+    e2e_t = torch.tensor([sum(e2e_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_value = pairs / (float(e2e_t[0]) / 1e3 / args.e2e_steps)
+
+    if rank == 0:
+        value = pairs / (step_total_ms / 1e3 / args.steps)
+        peaks, src = _peaks()
+        f_mhz = float(peaks.get("sm_max_mhz", 1965.0))
+        sms = torch.cuda.get_device_properties(dev).multi_processor_count
+        peak_ops = sms * 128 * f_mhz * 1e6  # lane-ops/s: 4 SMSP x 32 lanes x 1 warp-instr/clk
+        kern_s = kern_total_ms / 1e3 / args.steps
+        achieved = ops_alg / world / kern_s  # per-GPU kernel throughput (each rank runs 1/world of the ops)
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": step_total_ms / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": value / PAPER_GCD_PER_S, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": "cfg3: all-pairs 1024-bit RSA moduli, n=16384 (134,209,536 pairs), 8 planted "
+                                   "shared primes (BASELINE.json configs[2])",
+                       "n": n, "bits": bits, "pairs": pairs, "mode": "rsa-early-terminate",
+                       "parallelism": f"row-band x{world}" + (" + NCCL hit all-gather" if world > 1 else ""),
+                       "l2": "flushed before every step (256 MiB write); inputs 2 MiB",
+                       "ns_per_gcd": step_total_ms / args.steps * 1e6 / pairs,
+                       "iterations_per_gcd": iters / pairs, "limb_steps_per_gcd": limbs / pairs,
+                       "hits_ok": bool(ok), "hits": len(found), "wall_s": t_wall},
+            "roofline": {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
+                         "unit": "T int lane-ops/s", "frac": achieved / peak_ops, "traffic": _traffic(),
+                         "kernel": "allpairs_kernel<32>", "kernel_ms": kern_s * 1e3,
+                         "kernel_share_of_step": kern_total_ms / step_total_ms,
+                         "ops_per_gcd": ops_alg / pairs,
+                         "peak_source": f"{sms} SMs x 128 lanes x {f_mhz:.0f} MHz ({src} MEASURED_PEAKS sm_max_mhz)"},
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,
+                    "d2h_bytes_per_step": int(d2h) * world},
+            "gpu_launches": 2 * args.steps,
+            "clocks": clk.summary(),
+        }
+        if world == 1 and not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline(ms)
+        print(json.dumps(line))
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -125,9 +125,11 @@ uint64_t bulkgcd_cohort_count(size_t n);
 
 /*
  * bulkgcd_pairs on device data: d_A, d_B, d_G interleaved [W][m_pad];
- * d_iters (may be NULL): per-pair iteration counts; d_scratch: >= 4
- * unsigned long long of device memory ([2] = summed iterations and [3] = slow
- * steps when flags has BULKGCD_FLAG_STATS).  No validation of operand values.
+ * d_iters (may be NULL): per-pair iteration counts; d_scratch: >= 8
+ * unsigned long long of device memory, zeroed by the call ([2] = summed
+ * iterations, [3] = slow-path steps, [4] = limb-steps = sum of lX over all
+ * iterations, when flags has BULKGCD_FLAG_STATS or d_iters is given).  No
+ * validation of operand values.
  */
 int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G, size_t m, size_t m_pad,
                          uint32_t bits, int mode, uint32_t *d_iters, unsigned long long *d_scratch,
@@ -137,11 +139,11 @@ int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G
  * One GPU's share of the all-pairs search: cohorts [cohort_begin, cohort_end)
  * over moduli d_N (row-major, n*W) and d_N_blk (bulkgcd_layout_blocked).  Hit
  * records go to d_hits[h*(2+W) ...] = {i, j, g[0..W-1]} in completion order;
- * d_counters (>= 4 unsigned long long, device) is zeroed by the call, then
+ * d_counters (>= 8 unsigned long long, device) is zeroed by the call, then
  * [0] = number of hits found (records beyond hit_cap are counted but not
- * written: retry with a larger buffer), [2]/[3] = iteration/slow-step
- * counters with BULKGCD_FLAG_STATS.  Moduli must be odd and > 1 (not checked
- * here).
+ * written: retry with a larger buffer); with BULKGCD_FLAG_STATS, [2] = summed
+ * iterations, [3] = slow-path steps, [4] = limb-steps (sum of lX, the words
+ * each update pass covers).  Moduli must be odd and > 1 (not checked here).
  */
 int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t n, uint32_t bits,
                            uint64_t cohort_begin, uint64_t cohort_end, uint32_t *d_hits, uint64_t hit_cap,

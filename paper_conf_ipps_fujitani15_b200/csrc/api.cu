@@ -89,7 +89,7 @@ size_t pad32(size_t m) { return (m + 31) / 32 * 32; }
 template <int W>
 int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m, size_t m_pad, int mode,
                  uint32_t *d_iters, unsigned long long *scratch, unsigned flags, cudaStream_t st) {
-    CK(cudaMemsetAsync(scratch, 0, 4 * sizeof(unsigned long long), st));
+    CK(cudaMemsetAsync(scratch, 0, 8 * sizeof(unsigned long long), st));
     PairsArgs a{dA, dB, dG, m, m_pad, scratch + 1, d_iters, scratch + 2, W * 16};
     uint64_t cohorts = (m + 31) / 32;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * 4, (cohorts + 3) / 4);
@@ -109,7 +109,7 @@ int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m,
 template <int W>
 int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t c0, uint64_t c1, uint32_t *dHits,
                     uint64_t cap, unsigned long long *counters, unsigned flags, cudaStream_t st) {
-    CK(cudaMemsetAsync(counters, 0, 4 * sizeof(unsigned long long), st));
+    CK(cudaMemsetAsync(counters, 0, 8 * sizeof(unsigned long long), st));
     if (c1 <= c0) return 0;
     AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
     uint64_t warps = c1 - c0;
@@ -237,7 +237,7 @@ int bulkgcd_pairs_ex(const uint32_t *A, const uint32_t *B, size_t m, uint32_t bi
     CK(dAc.alloc(cm, st));
     CK(dBc.alloc(cm, st));
     CK(dGc.alloc(cm, st));
-    CK(dS.alloc(4 * sizeof(unsigned long long), st));
+    CK(dS.alloc(8 * sizeof(unsigned long long), st));
     if (iters) CK(dIt.alloc(m * 4, st));
     CK(cudaMemcpyAsync(dA.p, A, rm, cudaMemcpyHostToDevice, st));
     CK(cudaMemcpyAsync(dB.p, B, rm, cudaMemcpyHostToDevice, st));
@@ -283,7 +283,7 @@ int bulkgcd_all_pairs(const uint32_t *N, size_t n, uint32_t bits, bulkgcd_hits_t
     DBuf dN, dBlk, dC, dH;
     CK(dN.alloc(n * W * 4, st));
     CK(dBlk.alloc(bulkgcd_blocked_words(n, bits) * 4, st));
-    CK(dC.alloc(4 * sizeof(unsigned long long), st));
+    CK(dC.alloc(8 * sizeof(unsigned long long), st));
     CK(cudaMemcpyAsync(dN.p, N, n * W * 4, cudaMemcpyHostToDevice, st));
     if ((rc = bulkgcd_layout_blocked(dN.as<uint32_t>(), dBlk.as<uint32_t>(), n, bits, st))) return rc;
     uint64_t cap = 1024;

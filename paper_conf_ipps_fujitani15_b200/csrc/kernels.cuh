@@ -116,7 +116,7 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 template <int W, bool STATS, class Cond, class Sink>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, uint32_t &iters,
-                                            uint32_t &nslow) {
+                                            uint32_t &nslow, uint32_t &limbs) {
     int s = 0;
     int fix = 0;     // pending fix-up of the last iteration (hot_iter's code)
     int resume = 0;  // roles of the next iteration: 0 -> (X, Y) = (A, B), 1 -> (B, A)
@@ -156,8 +156,11 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         bool top = run && lX == W - s;
         if (__any_sync(FULL, need) || !__any_sync(FULL, top)) return 1;
         live = run;
+        if (STATS && run) {
+            ++iters;
+            limbs += lX;  // limb-steps: words of X the update pass covers
+        }
         fix = hot_iter<W>(X, Y, lX, tX, lY, tY, s, run);
-        if (STATS && run) ++iters;
         return __any_sync(FULL, fix != 0) ? 2 : 0;
     };
 
@@ -262,7 +265,7 @@ struct PairsArgs {
     uint64_t m, m_pad;
     unsigned long long *work;  // cohort cursor, zeroed by the host
     uint32_t *iters;           // optional per-pair iteration counts
-    unsigned long long *stats; // optional [sum iterations, slow steps]
+    unsigned long long *stats; // optional [sum iterations, slow steps, limb-steps]
     int half;
 };
 
@@ -315,7 +318,7 @@ struct PairsSinkRsa {
 template <int W, bool RSA, bool STATS>
 __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a) {
     const int lane = threadIdx.x & 31;
-    uint32_t iters = 0, nslow = 0;
+    uint32_t iters = 0, nslow = 0, limbs = 0;
     for (;;) {
         unsigned long long c = 0;
         if (lane == 0) c = atomicAdd(a.work, 1ull);
@@ -336,7 +339,7 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a)
             bool live = valid;
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkRsa<W> sink{a.G, i, a.m_pad};
-            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow);
+            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs);
         } else {
             int k2 = 0;
             bool known = false;
@@ -352,7 +355,7 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a)
             }
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkExact<W> sink{a.G, i, a.m_pad, k2, false, 0, 0};
-            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, iters, nslow);
+            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, iters, nslow, limbs);
             // 64-bit tail: Case 1 of approx (lX <= 2): alpha = X div Y, exactly (L127).
             if (sink.tail) {
                 uint64_t x = sink.x64, y = sink.y64;
@@ -362,7 +365,10 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a)
                     x = x - y * q;
                     if (x) x >>= __ffsll((long long)x) - 1;
                     if (x < y) { uint64_t t = x; x = y; y = t; }
-                    if (STATS) ++iters;
+                    if (STATS) {
+                        ++iters;
+                        limbs += (x >> 32) ? 2 : 1;
+                    }
                 }
                 uint32_t g[2] = {lo32(x), hi32(x)};
                 write_shifted<W>(a.G + i, a.m_pad, g, 2, sink.k2);
@@ -373,6 +379,7 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a)
     if (STATS && a.stats) {
         atomicAdd(&a.stats[0], (unsigned long long)iters);
         atomicAdd(&a.stats[1], (unsigned long long)nslow);
+        atomicAdd(&a.stats[2], (unsigned long long)limbs);
     }
 }
 
@@ -402,7 +409,7 @@ struct AllPairsArgs {
     uint32_t *hits;                // hit records [i, j, g[W]]
     uint64_t hit_cap;
     unsigned long long *hit_count;
-    unsigned long long *stats;     // optional [sum iterations, slow steps]
+    unsigned long long *stats;     // optional [sum iterations, slow steps, limb-steps]
     int half;
 };
 
@@ -441,7 +448,7 @@ template <int W, bool STATS>
 __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) allpairs_kernel(AllPairsArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t nb = (a.n + 31) / 32;
-    uint32_t iters = 0, nslow = 0;
+    uint32_t iters = 0, nslow = 0, limbs = 0;
     for (;;) {
         unsigned long long c = 0;
         if (lane == 0) c = atomicAdd(a.work, 1ull);
@@ -469,11 +476,12 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) allpairs_kernel(AllPairsA
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
-        euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow);
+        euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs);
     }
     if (STATS && a.stats) {
         atomicAdd(&a.stats[0], (unsigned long long)iters);
         atomicAdd(&a.stats[1], (unsigned long long)nslow);
+        atomicAdd(&a.stats[2], (unsigned long long)limbs);
     }
 }
 

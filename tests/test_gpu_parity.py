@@ -135,7 +135,7 @@ def _band_run(bg, ms, bits, c0, c1, cap):
     dB = torch.empty(bg.bulkgcd_blocked_words(ms.m, bits), dtype=torch.int32, device=dev)
     bg.bulkgcd_layout_blocked(dN, dB, ms.m, bits)
     dH = torch.zeros(max(cap, 1) * (2 + W), dtype=torch.int32, device=dev)
-    dC = torch.zeros(4, dtype=torch.int64, device=dev)
+    dC = torch.zeros(8, dtype=torch.int64, device=dev)
     bg.bulkgcd_all_pairs_band(dN, dB, ms.m, bits, c0, c1, dH, cap, dC, bg.FLAG_STATS)
     torch.cuda.synchronize()
     count = int(dC[0].item())
@@ -168,8 +168,9 @@ def test_all_pairs_stats_counters(bg, cfg1):
     total = bg.bulkgcd_cohort_count(cfg1.m)
     _, _, ctr = _band_run(bg, cfg1, 1024, 0, total, 16)
     N = synth.ints(cfg1.N)
-    want = sum(am.gcd_rsa(N[i], N[j], 1024).iterations for i in range(64) for j in range(i + 1, 64))
-    assert int(ctr[2]) == want
+    tr = [am.gcd_rsa(N[i], N[j], 1024) for i in range(64) for j in range(i + 1, 64)]
+    assert int(ctr[2]) == sum(t.iterations for t in tr)      # iterations (Table IV's unit)
+    assert int(ctr[4]) == sum(t.limb_steps for t in tr)      # limb-steps (the roofline's unit, M2)
 
 
 @pytest.mark.slow

@@ -20,7 +20,7 @@ dB = torch.empty(bg.bulkgcd_blocked_words(n, bits), dtype=torch.int32, device=de
 bg.bulkgcd_layout_blocked(dN, dB, n, bits)
 total = bg.bulkgcd_cohort_count(n)
 dH = torch.zeros(1024 * (2 + W), dtype=torch.int32, device=dev)
-dC = torch.zeros(4, dtype=torch.int64, device=dev)
+dC = torch.zeros(8, dtype=torch.int64, device=dev)
 for _ in range(reps):
     bg.bulkgcd_all_pairs_band(dN, dB, n, bits, 0, total, dH, 1024, dC, 0)
 torch.cuda.synchronize()

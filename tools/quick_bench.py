@@ -25,7 +25,7 @@ def time_allpairs(ms, bits, reps, stats=False):
     total = bg.bulkgcd_cohort_count(ms.m)
     cap = 4096
     dH = torch.zeros(cap * (2 + W), dtype=torch.int32, device=dev)
-    dC = torch.zeros(4, dtype=torch.int64, device=dev)
+    dC = torch.zeros(8, dtype=torch.int64, device=dev)
     # stats run
     bg.bulkgcd_all_pairs_band(dN, dB, ms.m, bits, 0, total, dH, cap, dC, bg.FLAG_STATS)
     torch.cuda.synchronize()
@@ -56,7 +56,7 @@ def time_pairs(m, bits, reps, mode):
     dAc = torch.empty(m_pad * W, dtype=torch.int32, device=dev)
     dBc = torch.empty(m_pad * W, dtype=torch.int32, device=dev)
     dGc = torch.empty(m_pad * W, dtype=torch.int32, device=dev)
-    dS = torch.zeros(4, dtype=torch.int64, device=dev)
+    dS = torch.zeros(8, dtype=torch.int64, device=dev)
     bg.bulkgcd_interleave(dA, dAc, m, m_pad, bits, True)
     bg.bulkgcd_interleave(dB, dBc, m, m_pad, bits, True)
     bg.bulkgcd_pairs_device(dAc, dBc, dGc, m, m_pad, bits, mode, None, dS, bg.FLAG_STATS)
