@@ -128,8 +128,8 @@ uint64_t bulkgcd_cohort_count(size_t n);
  * d_iters (may be NULL): per-pair iteration counts; d_scratch: >= 8
  * unsigned long long of device memory, zeroed by the call ([2] = summed
  * iterations, [3] = slow-path steps, [4] = limb-steps = sum of lX over all
- * iterations, when flags has BULKGCD_FLAG_STATS or d_iters is given).  No
- * validation of operand values.
+ * iterations, [5] = lane-slots, when flags has BULKGCD_FLAG_STATS or d_iters
+ * is given).  No validation of operand values.
  */
 int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G, size_t m, size_t m_pad,
                          uint32_t bits, int mode, uint32_t *d_iters, unsigned long long *d_scratch,
@@ -143,7 +143,8 @@ int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G
  * [0] = number of hits found (records beyond hit_cap are counted but not
  * written: retry with a larger buffer); with BULKGCD_FLAG_STATS, [2] = summed
  * iterations, [3] = slow-path steps, [4] = limb-steps (sum of lX, the words
- * each update pass covers).  Moduli must be odd and > 1 (not checked here).
+ * each update pass covers), [5] = lane-slots (32 x warp-iterations; [2]/[5]
+ * is the SIMT lane efficiency).  Moduli must be odd and > 1 (not checked here).
  */
 int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t n, uint32_t bits,
                            uint64_t cohort_begin, uint64_t cohort_end, uint32_t *d_hits, uint64_t hit_cap,

@@ -108,28 +108,33 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // finished lanes whose result needs the operand registers (sink), and the
 // realign when the warp length L dropped.  Keeping every conditional write of
 // the register arrays out of the hot loop stops ptxas from materialising
-// whole-array copies at merge points.
+// whole-array copies at merge points.  Each hot iteration ends with the loop
+// test of the next one, and all warp-level decisions of an iteration are one
+// redux.or: bit 0 = "some lane needs the cold section", bit 1 = "some running
+// lane still reaches the top register" (if none, the warp length L dropped and
+// the cold section realigns; this also covers "no lane running").
 //
 // Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
 // and returns true if a finished lane needs cold(...) (warp-converged, with
 // the operand registers); scalar-only finishes are handled by quick itself.
-template <int W, bool STATS, class Cond, class Sink>
+template <int W, bool STATS, bool EXACT, class Cond, class Sink>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, uint32_t &iters,
-                                            uint32_t &nslow, uint32_t &limbs) {
+                                            uint32_t &nslow, uint32_t &limbs, uint32_t &slots) {
     int s = 0;
     int fix = 0;     // pending fix-up of the last iteration (hot_iter's code)
     int resume = 0;  // roles of the next iteration: 0 -> (X, Y) = (A, B), 1 -> (B, A)
 
     // Cold section for the next roles (X, Y); the last iteration ran on (Y, X).
+    // Applies fix-ups, runs the loop test, serves finished lanes, realigns.
     auto cold = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
         if (__any_sync(FULL, fix != 0)) {
             if (STATS && fix >= 2) ++nslow;
             apply_fix<W>(fix, Y, X, lY, tY, lX, tX, s);
             fix = 0;
         }
-        bool run = live && cond(lX, tX, lY, tY);
-        bool fin = live && !run;
+        bool run = live & cond(lX, tX, lY, tY);
+        bool fin = live & !run;
         if (__any_sync(FULL, fin)) {
             bool need = sink.quick(fin, lX, tX, lY, tY);
             if (__any_sync(FULL, need)) sink.cold(need, X, Y, lX, tX, lY, tY, s);
@@ -144,46 +149,44 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         }
         return true;
     };
-    // One hot iteration on roles (X, Y).  0: continue; 1: go cold before the
-    // iteration (same roles); 2: iteration done, fix-ups pending (roles flip).
-    auto hot = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> int {
-        bool run = live && cond(lX, tX, lY, tY);
-        bool fin = live && !run;
-        bool need = sink.quick(fin, lX, tX, lY, tY);
-        // Go cold if a finished lane needs its registers, or if no running lane
-        // reaches the top register any more (the warp length L dropped: realign;
-        // this also covers "no lane running").  lX <= W - s always holds.
-        bool top = run && lX == W - s;
-        if (__any_sync(FULL, need) || !__any_sync(FULL, top)) return 1;
-        live = run;
-        if (STATS && run) {
-            ++iters;
-            limbs += lX;  // limb-steps: words of X the update pass covers
+    // One hot iteration on roles (X, Y) (its loop test already passed: the
+    // live lanes are the running ones), then the loop test of the next
+    // iteration (roles (Y, X)).  Returns true to go cold.
+    auto hot = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
+        if (STATS) {
+            ++slots;
+            if (live) {
+                ++iters;
+                limbs += lX;  // limb-steps: words of X the update pass covers
+            }
         }
-        fix = hot_iter<W>(X, Y, lX, tX, lY, tY, s, run);
-        return __any_sync(FULL, fix != 0) ? 2 : 0;
+        fix = hot_iter<W, EXACT>(X, Y, lX, tX, lY, tY, s, live);
+        bool run = live & cond(lY, tY, lX, tX);
+        bool fin = live & !run & (fix == 0);
+        bool need = sink.quick(fin, lY, tY, lX, tX) | (fix != 0);
+        bool top = run & (lY == W - s);
+        unsigned v = __reduce_or_sync(FULL, (need ? 1u : 0u) | (top ? 2u : 0u));
+        if (v != 2u) return true;
+        live = run;
+        return false;
     };
 
     for (;;) {
         bool more = resume == 0 ? cold(A, B, lA, tA, lB, tB) : cold(B, A, lB, tB, lA, tA);
         if (!more) return;
-        int rc;
         if (resume == 1) {
-            rc = hot(B, A, lB, tB, lA, tA);
-            if (rc) {
-                resume = rc == 2 ? 0 : 1;
+            if (hot(B, A, lB, tB, lA, tA)) {
+                resume = 0;
                 continue;
             }
         }
         for (;;) {
-            rc = hot(A, B, lA, tA, lB, tB);
-            if (rc) {
-                resume = rc == 2 ? 1 : 0;
+            if (hot(A, B, lA, tA, lB, tB)) {
+                resume = 1;
                 break;
             }
-            rc = hot(B, A, lB, tB, lA, tA);
-            if (rc) {
-                resume = rc == 2 ? 0 : 1;
+            if (hot(B, A, lB, tB, lA, tA)) {
+                resume = 0;
                 break;
             }
         }
@@ -203,7 +206,7 @@ struct RsaCond {
 // lX <= 2, finishes in the 64-bit tail).
 struct ExactCond {
     __device__ __forceinline__ bool operator()(int lX, uint64_t tX, int lY, uint64_t tY) const {
-        return lY >= 1 && lX >= 3;
+        return (lY >= 1) & (lX >= 3);
     }
 };
 
@@ -318,7 +321,7 @@ struct PairsSinkRsa {
 template <int W, bool RSA, bool STATS>
 __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a) {
     const int lane = threadIdx.x & 31;
-    uint32_t iters = 0, nslow = 0, limbs = 0;
+    uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0;
     for (;;) {
         unsigned long long c = 0;
         if (lane == 0) c = atomicAdd(a.work, 1ull);
@@ -339,7 +342,7 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a)
             bool live = valid;
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkRsa<W> sink{a.G, i, a.m_pad};
-            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs);
+            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs, slots);
         } else {
             int k2 = 0;
             bool known = false;
@@ -355,7 +358,7 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a)
             }
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkExact<W> sink{a.G, i, a.m_pad, k2, false, 0, 0};
-            euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, iters, nslow, limbs);
+            euclid_loop<W, STATS, true>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, iters, nslow, limbs, slots);
             // 64-bit tail: Case 1 of approx (lX <= 2): alpha = X div Y, exactly (L127).
             if (sink.tail) {
                 uint64_t x = sink.x64, y = sink.y64;
@@ -380,6 +383,7 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a)
         atomicAdd(&a.stats[0], (unsigned long long)iters);
         atomicAdd(&a.stats[1], (unsigned long long)nslow);
         atomicAdd(&a.stats[2], (unsigned long long)limbs);
+        atomicAdd(&a.stats[3], (unsigned long long)slots);  // lane-slots: warp-iterations x 32
     }
 }
 
@@ -448,7 +452,7 @@ template <int W, bool STATS>
 __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) allpairs_kernel(AllPairsArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t nb = (a.n + 31) / 32;
-    uint32_t iters = 0, nslow = 0, limbs = 0;
+    uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0;
     for (;;) {
         unsigned long long c = 0;
         if (lane == 0) c = atomicAdd(a.work, 1ull);
@@ -476,12 +480,13 @@ __global__ void __launch_bounds__(THREADS, MIN_BLOCKS) allpairs_kernel(AllPairsA
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
-        euclid_loop<W, STATS>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs);
+        euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs, slots);
     }
     if (STATS && a.stats) {
         atomicAdd(&a.stats[0], (unsigned long long)iters);
         atomicAdd(&a.stats[1], (unsigned long long)nslow);
         atomicAdd(&a.stats[2], (unsigned long long)limbs);
+        atomicAdd(&a.stats[3], (unsigned long long)slots);  // lane-slots: warp-iterations x 32
     }
 }
 
