@@ -160,13 +160,18 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
                 limbs += lX;  // limb-steps: words of X the update pass covers
             }
         }
-        fix = hot_iter<W, EXACT>(X, Y, lX, tX, lY, tY, s, live);
+        bool full, post, lt;
+        hot_iter<W, EXACT>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
+        bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
-        bool fin = live & !run & (fix == 0);
-        bool need = sink.quick(fin, lY, tY, lX, tX) | (fix != 0);
+        bool fin = live & !run & !bad;
+        bool need = sink.quick(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
         unsigned v = __reduce_or_sync(FULL, (need ? 1u : 0u) | (top ? 2u : 0u));
-        if (v != 2u) return true;
+        if (v != 2u) {
+            fix = fix_code(live, full, post, lt);
+            return true;
+        }
         live = run;
         return false;
     };
@@ -198,7 +203,8 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
 struct RsaCond {
     int half;
     __device__ __forceinline__ bool operator()(int lX, uint64_t tX, int lY, uint64_t tY) const {
-        return 32 * lY - (int)__clz(hi32(tY)) >= half;  // bitlen(Y); lY = 0 gives -32
+        // bitlen(Y) >= half (half a multiple of 32): lY > half/32, or lY == half/32 with y1's top bit set
+        return 2 * lY + (int)(hi32(tY) >> 31) > half / 16;
     }
 };
 
