@@ -92,7 +92,7 @@ int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m,
     CK(cudaMemsetAsync(scratch, 0, 8 * sizeof(unsigned long long), st));
     PairsArgs a{dA, dB, dG, m, m_pad, scratch + 1, d_iters, scratch + 2, W * 16};
     uint64_t cohorts = (m + 31) / 32;
-    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * 4, (cohorts + 3) / 4);
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (cohorts + 3) / 4);
     if (grid == 0) return 0;
     bool stats = (flags & BULKGCD_FLAG_STATS) || d_iters;
     if (mode == BULKGCD_MODE_RSA) {
@@ -113,7 +113,7 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if (c1 <= c0) return 0;
     AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
     uint64_t warps = c1 - c0;
-    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * 4, (warps + 3) / 4);
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + 3) / 4);
     if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, 0, st>>>(a);
     else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, 0, st>>>(a);
     CK(cudaGetLastError());

@@ -10,8 +10,14 @@ namespace bulkgcd {
 
 constexpr int THREADS = 128;  // 4 warps per CTA
 #ifndef MIN_BLOCKS
-#define MIN_BLOCKS 3  // CTAs per SM (3 -> <= 168 registers per thread, no spills)
+#define MIN_BLOCKS 3  // CTAs per SM for W <= 32 (3 -> <= 168 registers per thread, no spills)
 #endif
+// CTAs per SM by width: the operands take 2W registers per thread; W = 64
+// (2048-bit) needs ~200 registers, i.e. 2 CTAs (8 warps) per SM.
+template <int W>
+struct Occ {
+    static constexpr int blocks = W >= 64 ? 2 : MIN_BLOCKS;
+};
 
 // ------------------------------------------------------------------ layouts
 // Word-interleaved ("column-wise", PAPER.md L361 and Fig. 3) layouts: lane t of
@@ -325,7 +331,7 @@ struct PairsSinkRsa {
 };
 
 template <int W, bool RSA, bool STATS>
-__global__ void __launch_bounds__(THREADS, MIN_BLOCKS) pairs_kernel(PairsArgs a) {
+__global__ void __launch_bounds__(THREADS, Occ<W>::blocks) pairs_kernel(PairsArgs a) {
     const int lane = threadIdx.x & 31;
     uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0;
     for (;;) {
@@ -455,7 +461,7 @@ struct HitSink {
 };
 
 template <int W, bool STATS>
-__global__ void __launch_bounds__(THREADS, MIN_BLOCKS) allpairs_kernel(AllPairsArgs a) {
+__global__ void __launch_bounds__(THREADS, Occ<W>::blocks) allpairs_kernel(AllPairsArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t nb = (a.n + 31) / 32;
     uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0;

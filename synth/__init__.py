@@ -58,12 +58,38 @@ def _load():
     return _lib
 
 
+CACHE_DIR = os.environ.get("BULKGCD_SYNTH_CACHE", os.path.join("/tmp", "bulkgcd_synth_cache"))
+
+
 def primes(pbits: int, seed: int, first: int, count: int, nthreads: int | None = None) -> np.ndarray:
-    """Primes #first..#first+count-1 of stream `seed`, as uint32[count, pbits/32]."""
+    """Primes #first..#first+count-1 of stream `seed`, as uint32[count, pbits/32].
+
+    Large requests are memoised on disk (CACHE_DIR) purely to save generation
+    time; the content is a deterministic function of the arguments and is
+    regenerated identically when the cache is absent.  Set
+    BULKGCD_SYNTH_CACHE="" to disable."""
+    path = None
+    if CACHE_DIR and count >= 4096:
+        path = os.path.join(CACHE_DIR, f"primes_{pbits}_{seed}_{first}_{count}.npy")
+        if os.path.exists(path):
+            try:
+                arr = np.load(path)
+                if arr.shape == (count, pbits // 32) and arr.dtype == np.uint32:
+                    return arr
+            except (OSError, ValueError):
+                pass
     out = np.zeros((count, pbits // 32), dtype=np.uint32)
     nt = nthreads or os.cpu_count() or 1
     if _load().synth_primes(pbits, seed, first, count, out.ctypes.data, nt) != 0:
         raise RuntimeError("synth_primes failed")
+    if path is not None:
+        try:
+            os.makedirs(CACHE_DIR, exist_ok=True)
+            tmp = path + f".{os.getpid()}.npy"
+            np.save(tmp, out)
+            os.replace(tmp, path)
+        except OSError:
+            pass
     return out
 
 
