@@ -41,8 +41,19 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-PAPER_GCD_PER_S = 1.0 / 0.346e-6  # GTX 780 Ti, 1024-bit early-terminate, 16K all pairs
+# The paper's GTX 780 Ti, early-terminate, all pairs of 16K moduli (Table V):
+# 0.346 us/GCD at 1024 bits, 1.33 us/GCD at 2048 bits.  Same workload size as cfg3 / cfg4.
+PAPER_GCD_PER_S = {("cfg3", 1024): 1.0 / 0.346e-6, ("cfg4", 2048): 1.0 / 1.33e-6}
 METRIC = "1024-bit GCDs/sec (all-pairs)"
+WORKLOADS = {
+    "cfg1": "cfg1: all-pairs 1024-bit RSA moduli, n=64 (2,016 pairs), 3 planted shared primes (BASELINE.json configs[0])",
+    "cfg3": "cfg3: all-pairs 1024-bit RSA moduli, n=16384 (134,209,536 pairs), 8 planted shared primes "
+            "(BASELINE.json configs[2])",
+    "cfg4": "cfg4: all-pairs 2048-bit RSA moduli, n=16384 (134,209,536 pairs), 8 planted shared primes "
+            "(BASELINE.json configs[3])",
+    "cfg5": "cfg5: all-pairs 1024-bit RSA moduli, n=65536 (2,147,450,880 pairs), 33 planted shared primes "
+            "(BASELINE.json configs[4])",
+}
 UNIT = "GCD/s"
 OPS_PER_LIMB, OPS_PER_ITER = 4, 16  # SURVEY.md §8(d) M2; DESIGN.md §Roofline
 
@@ -57,6 +68,17 @@ def _peaks():
             return json.load(f), "measured"
     except OSError:
         return {"sm_max_mhz": 1965.0}, "fallback"
+
+
+def _int_issue_peak():
+    """Measured integer issue ceiling (tools/intpeak.cu on this pool's B200s,
+    profiles/r1_intpeak.json): ALU + IMAD mix, warp-instructions/clk/SM."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r1_intpeak.json")) as f:
+            d = json.load(f)
+        return float(d["ops"]["SHF+IMAD(alu+fma issue probe)"]["warp_inst_per_clk_per_sm_at_max_clock"])
+    except (OSError, ValueError, KeyError):
+        return None
 
 
 def _traffic():
@@ -180,7 +202,7 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": t_tot / args.steps * 1e3, "higher_is_better": True,
-        "scaling": "strong", "vs_baseline": v / PAPER_GCD_PER_S, "dtype": "u32", "data": "synthetic",
+        "scaling": "strong", "vs_baseline": v / PAPER_GCD_PER_S[("cfg3", 1024)], "dtype": "u32", "data": "synthetic",
         "config": {"workload": "cfg3: all-pairs 1024-bit RSA moduli, n=16384 (134,209,536 pairs), 8 planted",
                    "per_step_sample_pairs": per_step, "mode": "rsa-early-terminate (oracle: exact gcd + O3 map)"},
         "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
@@ -198,6 +220,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--workload", default="cfg3", choices=sorted(WORKLOADS))
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -221,14 +244,16 @@ def main():
     bg.bulkgcd_device_check()
 
     # ---- inputs: rank 0 generates the seeded moduli, NCCL broadcast to the others
-    bits = 1024
+    k = int(args.workload[3:])
+    bits = synth.CONFIGS[k]["bits"]
     W = bits // 32
+    metric = f"{bits}-bit GCDs/sec (all-pairs)"
     if rank == 0:
-        ms = synth.config_moduli(3)
+        ms = synth.config_moduli(k)
         N = ms.N
         truth = ms.truth
     else:
-        N = np.zeros((16384, W), np.uint32)
+        N = np.zeros((synth.CONFIGS[k]["m"], W), np.uint32)
         truth = None
     if world > 1:
         t = torch.from_numpy(N.view(np.int32)).to(dev)
@@ -337,15 +362,18 @@ def main():
         peaks, src = _peaks()
         f_mhz = float(peaks.get("sm_max_mhz", 1965.0))
         sms = torch.cuda.get_device_properties(dev).multi_processor_count
-        peak_ops = sms * 128 * f_mhz * 1e6  # lane-ops/s: 4 SMSP x 32 lanes x 1 warp-instr/clk
+        guide_ops = sms * 128 * f_mhz * 1e6  # lane-ops/s: 4 SMSP x 32 lanes x 1 warp-instr/clk (guide)
+        ipc = _int_issue_peak()
+        peak_ops = sms * 32 * ipc * f_mhz * 1e6 if ipc else guide_ops
         kern_s = kern_total_ms / 1e3 / args.steps
         achieved = ops_alg / world / kern_s  # per-GPU kernel throughput (each rank runs 1/world of the ops)
+        paper = PAPER_GCD_PER_S.get((args.workload, bits))
         line = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "metric": metric, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": step_total_ms / args.steps, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": value / PAPER_GCD_PER_S, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": "cfg3: all-pairs 1024-bit RSA moduli, n=16384 (134,209,536 pairs), 8 planted "
-                                   "shared primes (BASELINE.json configs[2])",
+            "scaling": "strong", "vs_baseline": value / paper if paper else None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": WORKLOADS[args.workload],
                        "n": n, "bits": bits, "pairs": pairs, "mode": "rsa-early-terminate",
                        "parallelism": f"row-band x{world}" + (" + NCCL hit all-gather" if world > 1 else ""),
                        "l2": "flushed before every step (256 MiB write); inputs 2 MiB",
@@ -354,10 +382,14 @@ def main():
                        "hits_ok": bool(ok), "hits": len(found), "wall_s": t_wall},
             "roofline": {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
                          "unit": "T int lane-ops/s", "frac": achieved / peak_ops, "traffic": _traffic(),
-                         "kernel": "allpairs_kernel<32>", "kernel_ms": kern_s * 1e3,
+                         "kernel": f"allpairs_kernel<{W}>", "kernel_ms": kern_s * 1e3,
                          "kernel_share_of_step": kern_total_ms / step_total_ms,
                          "ops_per_gcd": ops_alg / pairs,
-                         "peak_source": f"{sms} SMs x 128 lanes x {f_mhz:.0f} MHz ({src} MEASURED_PEAKS sm_max_mhz)"},
+                         "peak_source": (f"measured integer issue ceiling {ipc:.3f} warp-instr/clk/SM "
+                                         f"(profiles/r1_intpeak.json) x 32 lanes x {sms} SMs x {f_mhz:.0f} MHz "
+                                         f"({src} MEASURED_PEAKS sm_max_mhz)") if ipc else
+                                        f"{sms} SMs x 128 lanes x {f_mhz:.0f} MHz (guide unit counts)",
+                         "peak_guide": guide_ops / 1e12, "frac_of_guide_peak": achieved / guide_ops},
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,
                     "d2h_bytes_per_step": int(d2h) * world},
             "gpu_launches": 2 * args.steps,
