@@ -115,10 +115,10 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // realign when the warp length L dropped.  Keeping every conditional write of
 // the register arrays out of the hot loop stops ptxas from materialising
 // whole-array copies at merge points.  Each hot iteration ends with the loop
-// test of the next one, and all warp-level decisions of an iteration are one
-// redux.or: bit 0 = "some lane needs the cold section", bit 1 = "some running
+// test of the next one, and all warp-level decisions of an iteration are two
+// votes: "some lane needs the cold section" and "some running
 // lane still reaches the top register" (if none, the warp length L dropped and
-// the cold section realigns; this also covers "no lane running").
+// the cold section realigns; this also covers "no lane running") -- two ballots.
 //
 // Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
 // and returns true if a finished lane needs cold(...) (warp-converged, with
@@ -173,8 +173,8 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         bool fin = live & !run & !bad;
         bool need = sink.quick(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
-        unsigned v = __reduce_or_sync(FULL, (need ? 1u : 0u) | (top ? 2u : 0u));
-        if (v != 2u) {
+        unsigned bneed = __ballot_sync(FULL, need), btop = __ballot_sync(FULL, top);
+        if ((bneed != 0u) | (btop == 0u)) {
             fix = fix_code(live, full, post, lt);
             return true;
         }
