@@ -114,8 +114,15 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
     uint64_t warps = c1 - c0;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + 3) / 4);
-    if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, 0, st>>>(a);
-    else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, 0, st>>>(a);
+    constexpr size_t smem = allpairs_smem_bytes<W>();
+    static bool attr_done[2] = {false, false};  // idempotent, benign race
+    if (!attr_done[0]) {
+        CK(cudaFuncSetAttribute(allpairs_kernel<W, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        CK(cudaFuncSetAttribute(allpairs_kernel<W, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        attr_done[0] = true;
+    }
+    if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
+    else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, smem, st>>>(a);
     CK(cudaGetLastError());
     return 0;
 }

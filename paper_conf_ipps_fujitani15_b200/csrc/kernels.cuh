@@ -460,39 +460,121 @@ struct HitSink {
     }
 };
 
+// ---- TMA (bulk async copy) staging of a cohort's operands into shared memory
+// Per warp, a double buffer: while the warp runs cohort c, the copy engine
+// brings cohort c+1's row block (W x 32 words, one contiguous W*128-byte
+// block of the blocked layout) and column modulus (W words) into the other
+// buffer, completing on an mbarrier (cp.async.bulk ... mbarrier::complete_tx).
+template <int W>
+struct StageBuf {
+    uint32_t row[W * 32];
+    uint32_t col[W];
+};
+
+template <int W>
+constexpr size_t allpairs_smem_bytes() {
+    return (THREADS / 32) * 2 * sizeof(StageBuf<W>) + (THREADS / 32) * 2 * sizeof(unsigned long long);
+}
+
+__device__ __forceinline__ uint32_t smem_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long *bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, unsigned phase) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" ::"r"(smem_addr(bar)),
+        "r"(phase)
+        : "memory");
+}
+
+__device__ __forceinline__ void tma_bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long long *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_addr(dst)),
+        "l"(src), "r"(bytes), "r"(smem_addr(bar))
+        : "memory");
+}
+
+// cohort id -> (row block b, column j): largest b with P(b) <= c
+__device__ __forceinline__ void cohort_coords(uint64_t c, uint64_t n, uint64_t &b, uint64_t &j) {
+    uint64_t nb = (n + 31) / 32;
+    uint64_t lo = 0, hi = nb;  // P(lo) <= c < P(hi)
+    while (hi - lo > 1) {
+        uint64_t mid = (lo + hi) / 2;
+        if (cohorts_before(mid, n) <= c) lo = mid; else hi = mid;
+    }
+    b = lo;
+    j = 32 * b + 1 + (c - cohorts_before(b, n));
+}
+
 template <int W, bool STATS>
 __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) allpairs_kernel(AllPairsArgs a) {
-    const int lane = threadIdx.x & 31;
-    const uint64_t nb = (a.n + 31) / 32;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    StageBuf<W> *buf = reinterpret_cast<StageBuf<W> *>(smem_raw) + 2 * warp;
+    unsigned long long *bar =
+        reinterpret_cast<unsigned long long *>(smem_raw + (THREADS / 32) * 2 * sizeof(StageBuf<W>)) + 2 * warp;
+    if (lane == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
     uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0;
-    for (;;) {
-        unsigned long long c = 0;
-        if (lane == 0) c = atomicAdd(a.work, 1ull);
-        c = __shfl_sync(FULL, c, 0) + a.c_begin;
-        if (c >= a.c_end) break;
-        // cohort id -> (row block b, column j): largest b with P(b) <= c
-        uint64_t lo = 0, hi = nb;  // P(lo) <= c < P(hi)
-        while (hi - lo > 1) {
-            uint64_t mid = (lo + hi) / 2;
-            if (cohorts_before(mid, a.n) <= c) lo = mid; else hi = mid;
+    unsigned phase[2] = {0, 0};
+    constexpr unsigned kBytes = (W * 32 + W) * 4;
+
+    // claim a cohort and (lane 0) start its copy into buffer `slot`
+    auto claim = [&](int slot, uint64_t &c, uint64_t &b, uint64_t &j) -> bool {
+        unsigned long long cc = 0;
+        if (lane == 0) cc = atomicAdd(a.work, 1ull);
+        c = __shfl_sync(FULL, cc, 0) + a.c_begin;
+        if (c >= a.c_end) return false;
+        cohort_coords(c, a.n, b, j);
+        if (lane == 0) {
+            mbar_expect_tx(&bar[slot], kBytes);
+            tma_bulk_g2s(buf[slot].row, a.N_blk + b * W * 32, W * 32 * 4, &bar[slot]);
+            tma_bulk_g2s(buf[slot].col, a.N_rm + j * W, W * 4, &bar[slot]);
         }
-        uint64_t b = lo;
-        uint64_t j = 32 * b + 1 + (c - cohorts_before(b, a.n));
+        return true;
+    };
+
+    int slot = 0;
+    uint64_t c, b, j;
+    bool have = claim(0, c, b, j);
+    while (have) {
+        uint64_t c2, b2, j2;
+        bool have2 = claim(slot ^ 1, c2, b2, j2);  // prefetch the next cohort
+        mbar_wait(&bar[slot], phase[slot]);
+        phase[slot] ^= 1;
         uint64_t i = 32 * b + lane;
         bool live = i < j;
         uint32_t A[W], B[W];
-        const uint32_t *rowp = a.N_blk + b * W * 32 + lane;
-        const uint32_t *colp = a.N_rm + j * W;
 #pragma unroll
         for (int k = 0; k < W; ++k) {
-            A[k] = rowp[k * 32];
-            B[k] = colp[k];
+            A[k] = buf[slot].row[k * 32 + lane];  // conflict-free: one bank per lane
+            B[k] = buf[slot].col[k];              // broadcast
         }
+        __syncwarp();  // the buffer is refilled only after the next claim, i.e. after this read
         int lA, lB;
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
         euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs, slots);
+        slot ^= 1;
+        have = have2;
+        c = c2;
+        b = b2;
+        j = j2;
     }
     if (STATS && a.stats) {
         atomicAdd(&a.stats[0], (unsigned long long)iters);
