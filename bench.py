@@ -163,9 +163,14 @@ def cpu_baseline(ms, target_s: float = 12.0, seed: int = 7):
     t0 = time.perf_counter()
     oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
     dt = time.perf_counter() - t0
+    i1, j1 = sample(1 << 13)  # one core, for the per-core figure
+    t1 = time.perf_counter()
+    oracle.gcd_index_pairs(ms.N, i1, j1, nthreads=1)
+    dt1 = time.perf_counter() - t1
     return {"value": i.size / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "value_1core": i1.size / dt1, "us_per_gcd_1core": dt1 / i1.size * 1e6,
             "sample": f"{i.size} seeded random (i<j) pairs of the {ms.m}-moduli workload, exact classical Euclid "
-                      f"(Knuth D), {dt:.1f}s on {cores} threads"}
+                      f"(Knuth D), {dt:.1f}s on {cores} threads; 1-core figure on {i1.size} pairs"}
 
 
 def run_reference(args):

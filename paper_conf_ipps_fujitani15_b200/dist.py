@@ -79,6 +79,9 @@ def gather_hits(local: torch.Tensor, group=None) -> torch.Tensor:
     the largest count (the only cross-GPU traffic).  Returns every rank's
     records concatenated (unsorted), on local's device."""
     width = local.shape[1]
+    dev = local.device
+    if dist.get_backend(group) == "gloo" and local.is_cuda:  # gloo collectives run on host tensors
+        local = local.cpu()
     cnt = torch.tensor([local.shape[0]], dtype=torch.int64, device=local.device)
     world = dist.get_world_size(group)
     counts = [torch.zeros_like(cnt) for _ in range(world)]
@@ -86,12 +89,12 @@ def gather_hits(local: torch.Tensor, group=None) -> torch.Tensor:
     counts = [int(c.item()) for c in counts]
     m = max(counts)
     if m == 0:
-        return local.new_zeros((0, width))
+        return local.new_zeros((0, width)).to(dev)
     pad = local.new_zeros((m, width))
     pad[: local.shape[0]] = local
     parts = [torch.empty_like(pad) for _ in range(world)]
     dist.all_gather(parts, pad, group=group)
-    return torch.cat([p[:c] for p, c in zip(parts, counts)])
+    return torch.cat([p[:c] for p, c in zip(parts, counts)]).to(dev)
 
 
 def records_to_hits(rec: np.ndarray, bits: int) -> Hits:

@@ -194,3 +194,30 @@ def test_all_pairs_config3_full(bg):
     # planted pairs through the oracle, gcd by gcd
     for a, b, g in ms.truth:
         assert oracle.gcd(synth.to_int(ms.N[a]), synth.to_int(ms.N[b])) == g
+
+
+def _dist_worker(rank, world, port, out):
+    import os
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)  # one GPU on the test box: every rank shares it
+    from paper_conf_ipps_fujitani15_b200.dist import all_pairs_distributed
+    ms = synth.moduli(200, 1024, seed=77, n_planted_pairs=5, cliques=(3,))
+    hits = all_pairs_distributed(ms.N, 1024).as_list()
+    out[rank] = (hits == ms.truth, len(hits))
+    dist.destroy_process_group()
+
+
+def test_distributed_band_driver_on_one_gpu(bg):
+    """dist.all_pairs_distributed with 3 ranks (gloo exchange) sharing cuda:0:
+    bands + hit gather + merge reproduce the exact hit set on every rank."""
+    import socket
+    import torch.multiprocessing as mp
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    out = mp.Manager().dict()
+    mp.spawn(_dist_worker, args=(3, port, out), nprocs=3, join=True)
+    assert all(out[r][0] for r in range(3)), dict(out)
