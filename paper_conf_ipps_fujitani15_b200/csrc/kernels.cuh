@@ -14,6 +14,9 @@ constexpr int THREADS = 128;  // 4 warps per CTA
 #endif
 // CTAs per SM by width: the operands take 2W registers per thread; W = 64
 // (2048-bit) needs ~200 registers, i.e. 2 CTAs (8 warps) per SM.
+#ifndef BULKGCD_INLINE_REALIGN
+#define BULKGCD_INLINE_REALIGN 1
+#endif
 template <int W>
 struct Occ {
     static constexpr int blocks = W >= 64 ? 2 : MIN_BLOCKS;
@@ -174,10 +177,26 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         bool need = sink.quick(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
         unsigned bneed = __ballot_sync(FULL, need), btop = __ballot_sync(FULL, top);
+#if BULKGCD_INLINE_REALIGN
+        if (bneed != 0u) {
+            fix = fix_code(live, full, post, lt);
+            return true;
+        }
+        if (btop == 0u) {  // the warp length dropped: realign one word in place (or go cold if nobody runs)
+            if (__ballot_sync(FULL, run) == 0u) {
+                fix = 0;
+                return true;
+            }
+            shift_up_1<W>(A);
+            shift_up_1<W>(B);
+            ++s;
+        }
+#else
         if ((bneed != 0u) | (btop == 0u)) {
             fix = fix_code(live, full, post, lt);
             return true;
         }
+#endif
         live = run;
         return false;
     };
