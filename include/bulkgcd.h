@@ -144,7 +144,8 @@ int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G
  * written: retry with a larger buffer); with BULKGCD_FLAG_STATS, [2] = summed
  * iterations, [3] = slow-path steps, [4] = limb-steps (sum of lX, the words
  * each update pass covers), [5] = lane-slots (32 x warp-iterations; [2]/[5]
- * is the SIMT lane efficiency).  Moduli must be odd and > 1 (not checked here).
+ * is the SIMT lane efficiency), [6] = lane-words issued by the passes ([4]/[6]
+ * is the pass-word efficiency).  Moduli must be odd and > 1 (not checked here).
  */
 int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t n, uint32_t bits,
                            uint64_t cohort_begin, uint64_t cohort_end, uint32_t *d_hits, uint64_t hit_cap,

@@ -14,9 +14,6 @@ constexpr int THREADS = 128;  // 4 warps per CTA
 #endif
 // CTAs per SM by width: the operands take 2W registers per thread; W = 64
 // (2048-bit) needs ~200 registers, i.e. 2 CTAs (8 warps) per SM.
-#ifndef BULKGCD_INLINE_REALIGN
-#define BULKGCD_INLINE_REALIGN 1
-#endif
 template <int W>
 struct Occ {
     static constexpr int blocks = W >= 64 ? 2 : MIN_BLOCKS;
@@ -126,11 +123,12 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
 // and returns true if a finished lane needs cold(...) (warp-converged, with
 // the operand registers); scalar-only finishes are handled by quick itself.
-template <int W, bool STATS, bool EXACT, class Cond, class Sink>
+template <int W, bool STATS, bool EXACT, class Cond, class Sink, class Parker>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
-                                            uint64_t &tB, bool live, Cond cond, Sink &sink, uint32_t &iters,
-                                            uint32_t &nslow, uint32_t &limbs, uint32_t &slots) {
-    int s = 0;
+                                            uint64_t &tB, bool live, Cond cond, Sink &sink, Parker &pk, int s0,
+                                            uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
+                                            uint32_t &passw) {
+    int s = s0;
     int fix = 0;     // pending fix-up of the last iteration (hot_iter's code)
     int resume = 0;  // roles of the next iteration: 0 -> (X, Y) = (A, B), 1 -> (B, A)
 
@@ -149,7 +147,13 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
             if (__any_sync(FULL, need)) sink.cold(need, X, Y, lX, tX, lY, tY, s);
         }
         live = run;
-        if (!__any_sync(FULL, run)) return false;
+        unsigned brun = __ballot_sync(FULL, run);
+        if (brun == 0u) return false;
+        if (Parker::enabled && pk.wants(__popc(brun))) {  // few stragglers left: park them, free the warp
+            pk.park(run, brun, X, Y, lX, tX, lY, tY, s, sink);
+            live = false;
+            return false;
+        }
         int L = __reduce_max_sync(FULL, (unsigned)(run ? lX : 0));
         while (W - s > L) {
             shift_up_1<W>(A);
@@ -164,6 +168,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
     auto hot = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
         if (STATS) {
             ++slots;
+            passw += W - s;  // words the warp's pass covers this iteration
             if (live) {
                 ++iters;
                 limbs += lX;  // limb-steps: words of X the update pass covers
@@ -177,26 +182,22 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         bool need = sink.quick(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
         unsigned bneed = __ballot_sync(FULL, need), btop = __ballot_sync(FULL, top);
-#if BULKGCD_INLINE_REALIGN
         if (bneed != 0u) {
             fix = fix_code(live, full, post, lt);
             return true;
         }
-        if (btop == 0u) {  // the warp length dropped: realign one word in place (or go cold if nobody runs)
-            if (__ballot_sync(FULL, run) == 0u) {
-                fix = 0;
+        if (btop == 0u) {  // the warp length dropped (lanes finished or shrank): realign one word in place
+            unsigned brun = __ballot_sync(FULL, run);
+            // go cold if nobody runs, or to park the last few stragglers (checked only here:
+            // the warp length drops when the longest lanes finish)
+            if ((brun == 0u) | (Parker::enabled && pk.wants(__popc(brun)))) {
+                fix = fix_code(live, full, post, lt);
                 return true;
             }
             shift_up_1<W>(A);
             shift_up_1<W>(B);
             ++s;
         }
-#else
-        if ((bneed != 0u) | (btop == 0u)) {
-            fix = fix_code(live, full, post, lt);
-            return true;
-        }
-#endif
         live = run;
         return false;
     };
@@ -222,6 +223,61 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         }
     }
 }
+
+// ---- straggler parking (SIMT lane efficiency; SURVEY.md §7 H-d)
+// A lockstep cohort runs as long as its slowest lane: ~10% of lane-slots are
+// idle.  When at most K lanes are still running, the warp parks them in a
+// per-warp shared-memory pool (state: both operands, lengths, tops, i, j) and
+// takes new work; 32 parked lanes later run together as one cohort.
+struct NoPark {
+    static constexpr bool enabled = false;
+    __device__ __forceinline__ bool wants(unsigned) const { return false; }
+    template <int W, class Sink>
+    __device__ __forceinline__ void park(bool, unsigned, uint32_t (&)[W], uint32_t (&)[W], int, uint64_t, int,
+                                         uint64_t, int, Sink &) {}
+};
+
+template <int W>
+struct ParkPool {  // per warp, in shared memory; word-interleaved by slot (conflict-free)
+    uint32_t x[W * 32];
+    uint32_t y[W * 32];
+    uint32_t meta[8 * 32];  // lX, lY, tX.lo, tX.hi, tY.lo, tY.hi, i, j
+};
+
+template <int W>
+struct Parker {
+    static constexpr bool enabled = true;
+    ParkPool<W> *pool;
+    unsigned npool;  // warp-uniform
+    unsigned K;      // park when <= K lanes still run (0: never)
+    __device__ __forceinline__ bool wants(unsigned nrun) const { return nrun <= K && npool + nrun <= 32u; }
+    template <class Sink>
+    __device__ __forceinline__ void park(bool run, unsigned brun, uint32_t (&X)[W], uint32_t (&Y)[W], int lX,
+                                         uint64_t tX, int lY, uint64_t tY, int s, Sink &sink) {
+        const unsigned lane = threadIdx.x & 31;
+        unsigned slot = npool + __popc(brun & ((1u << lane) - 1u));
+        if (run) {
+#pragma unroll
+            for (int k = 0; k < W; ++k) {
+                if (k >= s) {
+                    pool->x[(k - s) * 32 + slot] = X[k];  // least significant word first
+                    pool->y[(k - s) * 32 + slot] = Y[k];
+                }
+            }
+            uint32_t *m = pool->meta + slot;
+            m[0] = (uint32_t)lX;
+            m[32] = (uint32_t)lY;
+            m[64] = lo32(tX);
+            m[96] = hi32(tX);
+            m[128] = lo32(tY);
+            m[160] = hi32(tY);
+            m[192] = sink.i;
+            m[224] = sink.j;
+        }
+        npool += __popc(brun);
+        __syncwarp();
+    }
+};
 
 // RSA-mode loop condition (early-terminate, L243/L251/L255): continue while Y
 // has at least s/2 bits.
@@ -352,7 +408,7 @@ struct PairsSinkRsa {
 template <int W, bool RSA, bool STATS>
 __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) pairs_kernel(PairsArgs a) {
     const int lane = threadIdx.x & 31;
-    uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0;
+    uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0, passw = 0;
     for (;;) {
         unsigned long long c = 0;
         if (lane == 0) c = atomicAdd(a.work, 1ull);
@@ -373,7 +429,9 @@ __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) pairs_kernel(PairsArg
             bool live = valid;
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkRsa<W> sink{a.G, i, a.m_pad};
-            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs, slots);
+            NoPark np;
+            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow, limbs,
+                                         slots, passw);
         } else {
             int k2 = 0;
             bool known = false;
@@ -389,7 +447,9 @@ __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) pairs_kernel(PairsArg
             }
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkExact<W> sink{a.G, i, a.m_pad, k2, false, 0, 0};
-            euclid_loop<W, STATS, true>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, iters, nslow, limbs, slots);
+            NoPark np;
+            euclid_loop<W, STATS, true>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, np, 0, iters, nslow, limbs, slots,
+                                        passw);
             // 64-bit tail: Case 1 of approx (lX <= 2): alpha = X div Y, exactly (L127).
             if (sink.tail) {
                 uint64_t x = sink.x64, y = sink.y64;
@@ -415,6 +475,7 @@ __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) pairs_kernel(PairsArg
         atomicAdd(&a.stats[1], (unsigned long long)nslow);
         atomicAdd(&a.stats[2], (unsigned long long)limbs);
         atomicAdd(&a.stats[3], (unsigned long long)slots);  // lane-slots: warp-iterations x 32
+        atomicAdd(&a.stats[4], (unsigned long long)passw);  // lane-words of pass issued
     }
 }
 
@@ -490,9 +551,20 @@ struct StageBuf {
     uint32_t col[W];
 };
 
+#ifndef BULKGCD_PARK_K
+#define BULKGCD_PARK_K 0  // straggler parking: measured a wash on B200, off by default
+#endif
+// Parking pool only where it fits next to the TMA buffers at the kernel's occupancy.
+template <int W>
+struct ParkCfg {
+    static constexpr bool on = (W <= 32) && (BULKGCD_PARK_K > 0);
+    static constexpr size_t pool_bytes = on ? sizeof(ParkPool<W>) : 0;
+};
+
 template <int W>
 constexpr size_t allpairs_smem_bytes() {
-    return (THREADS / 32) * 2 * sizeof(StageBuf<W>) + (THREADS / 32) * 2 * sizeof(unsigned long long);
+    return (THREADS / 32) * (2 * sizeof(StageBuf<W>) + ParkCfg<W>::pool_bytes) +
+           (THREADS / 32) * 2 * sizeof(unsigned long long);
 }
 
 __device__ __forceinline__ uint32_t smem_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -540,15 +612,17 @@ __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) allpairs_kernel(AllPa
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     StageBuf<W> *buf = reinterpret_cast<StageBuf<W> *>(smem_raw) + 2 * warp;
+    unsigned char *after_bufs = smem_raw + (THREADS / 32) * 2 * sizeof(StageBuf<W>);
+    ParkPool<W> *pool = reinterpret_cast<ParkPool<W> *>(after_bufs) + warp;  // valid only if ParkCfg<W>::on
     unsigned long long *bar =
-        reinterpret_cast<unsigned long long *>(smem_raw + (THREADS / 32) * 2 * sizeof(StageBuf<W>)) + 2 * warp;
+        reinterpret_cast<unsigned long long *>(after_bufs + (THREADS / 32) * ParkCfg<W>::pool_bytes) + 2 * warp;
     if (lane == 0) {
         mbar_init(&bar[0], 1);
         mbar_init(&bar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncwarp();
-    uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0;
+    uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0, passw = 0;
     unsigned phase[2] = {0, 0};
     constexpr unsigned kBytes = (W * 32 + W) * 4;
 
@@ -567,10 +641,50 @@ __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) allpairs_kernel(AllPa
         return true;
     };
 
+    Parker<W> pk{pool, 0u, ParkCfg<W>::on ? (unsigned)BULKGCD_PARK_K : 0u};
+
+    // Run up to 32 parked stragglers as one cohort (top slots of the pool).
+    auto run_parked = [&](bool allow_park) {
+        unsigned take = pk.npool < 32u ? pk.npool : 32u;
+        unsigned slot = pk.npool - take + lane;
+        bool live = (unsigned)lane < take;
+        const uint32_t *m = pool->meta + slot;
+        int lA = live ? (int)m[0] : 0, lB = live ? (int)m[32] : 0;
+        uint64_t tA = live ? ((uint64_t)m[96] << 32 | m[64]) : 0, tB = live ? ((uint64_t)m[160] << 32 | m[128]) : 0;
+        uint32_t pi = live ? m[192] : 0u, pj = live ? m[224] : 0u;
+        int L = (int)__reduce_max_sync(FULL, (unsigned)lA);
+        int s = W - L;
+        uint32_t A[W], B[W];
+#pragma unroll
+        for (int k = 0; k < W; ++k) {  // pool words beyond a lane's own lengths are stale: read as zero
+            A[k] = (live & (k >= s) & (k - s < lA)) ? pool->x[(k - s) * 32 + slot] : 0u;
+            B[k] = (live & (k >= s) & (k - s < lB)) ? pool->y[(k - s) * 32 + slot] : 0u;
+        }
+        __syncwarp();
+        pk.npool -= take;
+        unsigned K = pk.K;
+        if (!allow_park) pk.K = 0;
+        HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, pi, pj};
+        euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
+                                     slots, passw);
+        pk.K = K;
+    };
+
     int slot = 0;
     uint64_t c, b, j;
     bool have = claim(0, c, b, j);
-    while (have) {
+    for (;;) {
+        if (ParkCfg<W>::on && pk.npool >= 32u) {
+            run_parked(true);
+            continue;
+        }
+        if (!have) {
+            if (ParkCfg<W>::on && pk.npool > 0u) {  // drain: no more fresh work
+                run_parked(false);
+                continue;
+            }
+            break;
+        }
         uint64_t c2, b2, j2;
         bool have2 = claim(slot ^ 1, c2, b2, j2);  // prefetch the next cohort
         mbar_wait(&bar[slot], phase[slot]);
@@ -588,7 +702,14 @@ __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) allpairs_kernel(AllPa
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
-        euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, iters, nslow, limbs, slots);
+        if (ParkCfg<W>::on) {
+            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
+                                         limbs, slots, passw);
+        } else {
+            NoPark np;
+            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
+                                         limbs, slots, passw);
+        }
         slot ^= 1;
         have = have2;
         c = c2;
@@ -600,6 +721,7 @@ __global__ void __launch_bounds__(THREADS, Occ<W>::blocks) allpairs_kernel(AllPa
         atomicAdd(&a.stats[1], (unsigned long long)nslow);
         atomicAdd(&a.stats[2], (unsigned long long)limbs);
         atomicAdd(&a.stats[3], (unsigned long long)slots);  // lane-slots: warp-iterations x 32
+        atomicAdd(&a.stats[4], (unsigned long long)passw);  // lane-words of pass issued
     }
 }
 

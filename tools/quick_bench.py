@@ -32,7 +32,8 @@ def time_allpairs(ms, bits, reps, stats=False):
     ctr = dC.cpu().numpy()
     pairs = ms.m * (ms.m - 1) // 2
     print(f"  hits={ctr[0]} truth={len(ms.truth)} iters/pair={ctr[2] / pairs:.2f} slow/pair={ctr[3] / pairs:.4f} "
-          f"limbs/pair={ctr[4] / pairs:.1f} simt_eff={ctr[2] / max(ctr[5], 1):.4f}")
+          f"limbs/pair={ctr[4] / pairs:.1f} simt_eff={ctr[2] / max(ctr[5], 1):.4f} "
+          f"word_eff={ctr[4] / max(ctr[6], 1):.4f} warp_iters/pair={ctr[5] / 32 / pairs:.3f}")
     ts = []
     for _ in range(reps):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
