@@ -42,7 +42,7 @@ __global__ void interleave_kernel(const uint32_t *__restrict__ in, uint32_t *__r
         } else {  // read interleaved: word k0+r, item i0+tx
             uint64_t i = i0 + tx;
             int k = k0 + r;
-            tile[tx][r] = (i < m_pad && k < W) ? in[(uint64_t)k * m_pad + i] : 0u;
+            tile[tx][r] = (i < m && k < W) ? in[(uint64_t)k * m_pad + i] : 0u;  // padding items are never read
         }
     }
     __syncthreads();
