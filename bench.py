@@ -58,6 +58,28 @@ UNIT = "GCD/s"
 OPS_PER_LIMB, OPS_PER_ITER = 4, 16  # SURVEY.md §8(d) M2; DESIGN.md §Roofline
 
 
+BACKEND = os.environ.get("BULKGCD_BENCH_BACKEND", "nccl")  # "gloo": test mode, ranks may share one GPU
+
+
+def _coll(fn, *tensors, **kw):
+    """Run a torch.distributed collective; with gloo, on host copies of device tensors."""
+    if BACKEND != "gloo":
+        return fn(*tensors, **kw)
+    host = [t.cpu() for t in tensors]
+    fn(*host, **kw)
+    for t, h in zip(tensors, host):
+        t.copy_(h)
+
+
+def _allgather_into(out, inp):
+    import torch.distributed as dist
+    if BACKEND != "gloo":
+        return dist.all_gather_into_tensor(out, inp)
+    parts = [inp.new_empty(inp.shape).cpu() for _ in range(dist.get_world_size())]
+    dist.all_gather(parts, inp.cpu())
+    out.copy_(__import__("torch").cat(parts))
+
+
 def _env_rank():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
@@ -242,10 +264,14 @@ def main():
     rank, world, local = _env_rank()
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world} (launch N>1 with torchrun)")
+    local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if BACKEND == "gloo":
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     bg.bulkgcd_device_check()
 
     # ---- inputs: rank 0 generates the seeded moduli, NCCL broadcast to the others
@@ -262,7 +288,7 @@ def main():
         truth = None
     if world > 1:
         t = torch.from_numpy(N.view(np.int32)).to(dev)
-        dist.broadcast(t, 0)
+        _coll(dist.broadcast, t, src=0)
         N = t.cpu().numpy().view(np.uint32)
     n = N.shape[0]
     pairs = n * (n - 1) // 2
@@ -281,8 +307,8 @@ def main():
         k1.record()
         if world > 1:
             # the exchange step: NCCL all-gather of the hit counts and fixed-capacity hit buffers
-            dist.all_gather_into_tensor(gcnt, runner.d_ctr[:1])
-            dist.all_gather_into_tensor(gbuf, runner.d_hits)
+            _allgather_into(gcnt, runner.d_ctr[:1])
+            _allgather_into(gbuf, runner.d_hits)
 
     # ---- algorithmic work of one launch (stats pass, untimed)
     runner.layout()
@@ -292,7 +318,7 @@ def main():
     iters, limbs = int(ctr[2]), int(ctr[4])
     if world > 1:
         tt = torch.tensor([iters, limbs], dtype=torch.int64, device=dev)
-        dist.all_reduce(tt)
+        _coll(dist.all_reduce, tt)
         iters, limbs = int(tt[0]), int(tt[1])
     ops_alg = OPS_PER_LIMB * limbs + OPS_PER_ITER * iters  # whole job, per step
 
@@ -337,7 +363,7 @@ def main():
 
     tot_ms = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
     if world > 1:
-        dist.all_reduce(tot_ms, op=dist.ReduceOp.MAX)
+        _coll(dist.all_reduce, tot_ms, op=dist.ReduceOp.MAX)
     step_total_ms, kern_total_ms = float(tot_ms[0]), float(tot_ms[1])
 
     # ---- end to end through the public API with host buffers
@@ -359,7 +385,7 @@ def main():
         e2e_ms.append(dt * 1e3)
     e2e_t = torch.tensor([sum(e2e_ms)], dtype=torch.float64, device=dev)
     if world > 1:
-        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        _coll(dist.all_reduce, e2e_t, op=dist.ReduceOp.MAX)
     e2e_value = pairs / (float(e2e_t[0]) / 1e3 / args.e2e_steps)
 
     if rank == 0:

@@ -221,3 +221,29 @@ def test_distributed_band_driver_on_one_gpu(bg):
     out = mp.Manager().dict()
     mp.spawn(_dist_worker, args=(3, port, out), nprocs=3, join=True)
     assert all(out[r][0] for r in range(3)), dict(out)
+
+
+def test_bench_multirank_path_gloo(bg):
+    """bench.py's N > 1 code path (torchrun, band split, hit exchange, max-over-ranks
+    timing) on the single test GPU, with gloo standing in for NCCL."""
+    import json
+    import os
+    import socket
+    import subprocess
+    import sys
+    from conftest import ROOT
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    env = dict(os.environ, BULKGCD_BENCH_BACKEND="gloo")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--workload", "cfg1", "--steps", "3", "--warmup", "3", "--no-cpu-baseline",
+           "--e2e-steps", "1"]
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    rec = json.loads(lines[0])
+    assert rec["n_gpus"] == 2 and rec["config"]["hits_ok"] and rec["config"]["hits"] == 3
+    assert rec["value"] > 0 and rec["e2e"]["value"] > 0
