@@ -151,6 +151,27 @@ int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t 
                            uint64_t cohort_begin, uint64_t cohort_end, uint32_t *d_hits, uint64_t hit_cap,
                            unsigned long long *d_counters, unsigned flags, void *stream);
 
+/*
+ * Factor output: "if gcd(n1, n2) = p != 1
+ * then n1 = p * (n1/p)".  For every hit h of a bulkgcd_all_pairs result on the
+ * same N and bits, F[(2h)*W + k] = word k of N[i] / g and F[(2h+1)*W + k] =
+ * word k of N[j] / g (exact division by the odd g, on the GPU).
+ * N: host row-major n*W words; F: host, caller-allocated, 2*count*W words.
+ * Errors: EINVAL (null pointer with count > 0, bits mismatch, an index >= n, or
+ * a g that is zero, even or does not divide its modulus), ENOMEM, ECUDA, ENODEV.
+ */
+int bulkgcd_cofactors(const uint32_t *N, size_t n, uint32_t bits, const bulkgcd_hits_t *hits, uint32_t *F);
+
+/*
+ * Device form: d_hits holds `count` records {i, j, g[W]} (the layout
+ * bulkgcd_all_pairs_band writes), d_F receives 2*count*W words as above, and
+ * *d_bad (device, zeroed by the caller) is incremented once per cofactor whose
+ * record is invalid or whose g does not divide the modulus (that F row is then
+ * meaningless).  Asynchronous on `stream`.
+ */
+int bulkgcd_cofactors_device(const uint32_t *d_N, size_t n, uint32_t bits, const uint32_t *d_hits, uint64_t count,
+                             uint32_t *d_F, unsigned long long *d_bad, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

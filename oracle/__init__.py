@@ -159,3 +159,17 @@ def all_pairs_hits(N: np.ndarray, bits: int, ii=None, jj=None, nthreads: int | N
     out = [(int(ii[k]), int(jj[k]), _int(G[k])) for k in np.nonzero(hit)[0]]
     out.sort()
     return out
+
+
+def cofactors(N: np.ndarray, hits) -> list[tuple[int, int]]:
+    """Factor output (n1 = p * (n1 / p)): for each hit (i, j, g),
+    (N[i] div g, N[j] div g) by the oracle's Knuth-D division; raises if g does
+    not divide a modulus (remainder != 0)."""
+    out = []
+    for i, j, g in hits:
+        qi, ri = divmod_(_int(np.asarray(N[i])), g)
+        qj, rj = divmod_(_int(np.asarray(N[j])), g)
+        if ri or rj:
+            raise ValueError(f"gcd does not divide N[{i}] or N[{j}]")
+        out.append((qi, qj))
+    return out

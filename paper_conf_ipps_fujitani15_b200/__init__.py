@@ -7,7 +7,8 @@ binding's functions raises.
 
 Names follow the C ABI: bulkgcd_pairs, bulkgcd_pairs_ex, bulkgcd_all_pairs,
 bulkgcd_interleave, bulkgcd_layout_blocked, bulkgcd_cohort_count,
-bulkgcd_blocked_words, bulkgcd_pairs_device, bulkgcd_all_pairs_band.
+bulkgcd_blocked_words, bulkgcd_pairs_device, bulkgcd_all_pairs_band,
+bulkgcd_cofactors, bulkgcd_cofactors_device.
 """
 from __future__ import annotations
 
@@ -31,6 +32,7 @@ SYMBOLS = (
     "bulkgcd_pairs", "bulkgcd_pairs_ex", "bulkgcd_all_pairs", "bulkgcd_hits_free", "bulkgcd_strerror",
     "bulkgcd_last_error", "bulkgcd_device_check", "bulkgcd_interleave", "bulkgcd_layout_blocked",
     "bulkgcd_blocked_words", "bulkgcd_cohort_count", "bulkgcd_pairs_device", "bulkgcd_all_pairs_band",
+    "bulkgcd_cofactors", "bulkgcd_cofactors_device",
 )
 
 
@@ -68,6 +70,8 @@ def lib() -> ctypes.CDLL:
             "bulkgcd_cohort_count": ([sz], u64),
             "bulkgcd_pairs_device": ([vp, vp, vp, sz, sz, u32, i32, vp, vp, ctypes.c_uint, vp], i32),
             "bulkgcd_all_pairs_band": ([vp, vp, sz, u32, u64, u64, vp, u64, vp, ctypes.c_uint, vp], i32),
+            "bulkgcd_cofactors": ([vp, sz, u32, ctypes.POINTER(_Hits), vp], i32),
+            "bulkgcd_cofactors_device": ([vp, sz, u32, vp, u64, vp, vp, vp], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -159,6 +163,21 @@ def bulkgcd_all_pairs(N, bits: int) -> Hits:
     return Hits(ij, g, bits)
 
 
+def bulkgcd_cofactors(N, bits: int, hits: Hits) -> np.ndarray:
+    """Factor output: F[h, 0] = N[i] / g, F[h, 1] = N[j] / g for
+    every hit (i, j, g), as uint32[count, 2, W] (exact division on the GPU)."""
+    W = _words(bits)
+    N = _host(N, W)
+    c = len(hits.ij)
+    ij = np.ascontiguousarray(hits.ij, dtype=np.uint32).reshape(c, 2)
+    g = np.ascontiguousarray(hits.gcd, dtype=np.uint32).reshape(c, W)
+    h = _Hits(c, ij.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)) if c else None,
+              g.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)) if c else None, hits.bits)
+    F = np.zeros((c, 2, W), np.uint32)
+    _check(lib().bulkgcd_cofactors(N.ctypes.data, N.shape[0], bits, ctypes.byref(h), F.ctypes.data))
+    return F
+
+
 def bulkgcd_device_check() -> None:
     _check(lib().bulkgcd_device_check())
 
@@ -191,3 +210,8 @@ def bulkgcd_all_pairs_band(d_N, d_N_blk, n: int, bits: int, cohort_begin: int, c
                            hit_cap: int, d_counters, flags: int = 0, stream=None) -> None:
     _check(lib().bulkgcd_all_pairs_band(_ptr(d_N), _ptr(d_N_blk), n, bits, cohort_begin, cohort_end,
                                         _ptr(d_hits), hit_cap, _ptr(d_counters), flags, _stream(stream)))
+
+
+def bulkgcd_cofactors_device(d_N, n: int, bits: int, d_hits, count: int, d_F, d_bad, stream=None) -> None:
+    _check(lib().bulkgcd_cofactors_device(_ptr(d_N), n, bits, _ptr(d_hits), count, _ptr(d_F), _ptr(d_bad),
+                                          _stream(stream)))

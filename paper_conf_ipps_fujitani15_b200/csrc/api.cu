@@ -14,6 +14,7 @@
 #include <vector>
 
 #include "../../include/bulkgcd.h"
+#include "factor.cuh"
 #include "kernels.cuh"
 
 using namespace bulkgcd;
@@ -336,6 +337,62 @@ int bulkgcd_all_pairs(const uint32_t *N, size_t n, uint32_t bits, bulkgcd_hits_t
     }
     out->count = count;
     out->bits = bits;
+    return 0;
+}
+
+int bulkgcd_cofactors_device(const uint32_t *d_N, size_t n, uint32_t bits, const uint32_t *d_hits, uint64_t count,
+                             uint32_t *d_F, unsigned long long *d_bad, void *stream) {
+    int W = words_for(bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u", bits);
+    if (count == 0) return 0;
+    if (!d_N || !d_hits || !d_F || !d_bad) return set_err(BULKGCD_EINVAL, "null pointer with count > 0");
+    cudaStream_t st = (cudaStream_t)stream;
+    uint64_t threads = 2 * count, block = 128, grid = (threads + block - 1) / block;
+    switch (W) {
+        case 16: cofactor_kernel<16><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
+        case 32: cofactor_kernel<32><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
+        default: cofactor_kernel<64><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
+    }
+    CK(cudaGetLastError());
+    return 0;
+}
+
+int bulkgcd_cofactors(const uint32_t *N, size_t n, uint32_t bits, const bulkgcd_hits_t *hits, uint32_t *F) {
+    int W = words_for(bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048)", bits);
+    if (!hits) return set_err(BULKGCD_EINVAL, "null hits");
+    if (hits->bits != bits) return set_err(BULKGCD_EINVAL, "hits were computed for %u bits, not %u", hits->bits, bits);
+    size_t count = hits->count;
+    if (count == 0) return 0;
+    if (!N || !F || !hits->ij || !hits->gcd) return set_err(BULKGCD_EINVAL, "null pointer with count > 0");
+    for (size_t h = 0; h < count; ++h)
+        if (hits->ij[h][0] >= n || hits->ij[h][1] >= n)
+            return set_err(BULKGCD_EINVAL, "hit %zu indexes a modulus >= n = %zu", h, n);
+    int rc = device_check();
+    if (rc) return rc;
+    cudaStream_t st = cudaStreamPerThread;
+    std::vector<uint32_t> rec(count * (2 + W));
+    for (size_t h = 0; h < count; ++h) {
+        rec[h * (2 + W)] = hits->ij[h][0];
+        rec[h * (2 + W) + 1] = hits->ij[h][1];
+        memcpy(&rec[h * (2 + W) + 2], hits->gcd + h * W, W * 4);
+    }
+    DBuf dN, dH, dF, dBad;
+    CK(dN.alloc(n * W * 4, st));
+    CK(dH.alloc(rec.size() * 4, st));
+    CK(dF.alloc(2 * count * W * 4, st));
+    CK(dBad.alloc(sizeof(unsigned long long), st));
+    CK(cudaMemcpyAsync(dN.p, N, n * W * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(dH.p, rec.data(), rec.size() * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemsetAsync(dBad.p, 0, sizeof(unsigned long long), st));
+    if ((rc = bulkgcd_cofactors_device(dN.as<uint32_t>(), n, bits, dH.as<uint32_t>(), count, dF.as<uint32_t>(),
+                                       dBad.as<unsigned long long>(), st)))
+        return rc;
+    unsigned long long bad = 0;
+    CK(cudaMemcpyAsync(F, dF.p, 2 * count * W * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&bad, dBad.p, sizeof bad, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (bad) return set_err(BULKGCD_EINVAL, "%llu cofactor(s): gcd is zero, even, or does not divide the modulus", bad);
     return 0;
 }
 

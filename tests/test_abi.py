@@ -60,6 +60,16 @@ def test_host_validation_no_gpu_needed(bg):
     one = np.zeros((1, W), np.uint32)
     one[0, 0] = 3
     assert bg.bulkgcd_all_pairs(one, 1024).ij.shape == (0, 2)
+    # cofactors: bits mismatch / index out of range are rejected on the host; no hits is a no-op
+    h = bg.Hits(np.array([[0, 1]], np.uint32), np.ones((1, W), np.uint32), 2048)
+    with pytest.raises(bg.BulkGcdError) as e:
+        bg.bulkgcd_cofactors(Z, 1024, h)
+    assert e.value.code == bg.EINVAL
+    h = bg.Hits(np.array([[0, 2]], np.uint32), np.ones((1, W), np.uint32), 1024)
+    with pytest.raises(bg.BulkGcdError) as e:
+        bg.bulkgcd_cofactors(Z, 1024, h)
+    assert e.value.code == bg.EINVAL
+    assert bg.bulkgcd_cofactors(Z, 1024, bg.Hits(h.ij[:0], h.gcd[:0], 1024)).shape == (0, 2, W)
 
 
 def test_cohort_enumeration(bg):

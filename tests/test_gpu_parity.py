@@ -128,6 +128,34 @@ def test_all_pairs_errors(bg, cfg1):
     assert bg.bulkgcd_all_pairs(cfg1.N[:1], 1024).ij.shape == (0, 2)
 
 
+@pytest.mark.parametrize("n,bits", [(40, 1024), (37, 512), (36, 2048)])
+def test_cofactors_factor_output(bg, n, bits):
+    """N3: exact division of both moduli of every hit by g (GPU) == the oracle's
+    Knuth-D quotients == the construction's other primes."""
+    ms = synth.moduli(n, bits, seed=n + bits, n_planted_pairs=2, cliques=(3,), n_duplicates=1)
+    hits = bg.bulkgcd_all_pairs(ms.N, bits)
+    assert hits.as_list() == ms.truth
+    F = bg.bulkgcd_cofactors(ms.N, bits, hits)
+    got = [(synth.to_int(F[h, 0]), synth.to_int(F[h, 1])) for h in range(F.shape[0])]
+    assert got == oracle.cofactors(ms.N, ms.truth)
+
+
+def test_cofactors_errors(bg, cfg1):
+    hits = bg.bulkgcd_all_pairs(cfg1.N, 1024)
+    assert bg.bulkgcd_cofactors(cfg1.N, 1024, bg.Hits(hits.ij[:0], hits.gcd[:0], 1024)).shape == (0, 2, 32)
+    bad = bg.Hits(hits.ij.copy(), hits.gcd.copy(), 1024)
+    bad.gcd[0, 0] += 2  # odd, but no longer a divisor
+    with pytest.raises(bg.BulkGcdError) as e:
+        bg.bulkgcd_cofactors(cfg1.N, 1024, bad)
+    assert e.value.code == bg.EINVAL
+    bad = bg.Hits(hits.ij.copy(), hits.gcd.copy(), 1024)
+    bad.ij[0, 1] = cfg1.m
+    with pytest.raises(bg.BulkGcdError):
+        bg.bulkgcd_cofactors(cfg1.N, 1024, bad)
+    with pytest.raises(bg.BulkGcdError):
+        bg.bulkgcd_cofactors(cfg1.N, 1024, bg.Hits(hits.ij, hits.gcd, 2048))
+
+
 def _band_run(bg, ms, bits, c0, c1, cap):
     W = bits // 32
     dev = torch.device("cuda")

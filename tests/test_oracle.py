@@ -135,3 +135,19 @@ def test_rsa_mode_mapping():
     G = synth.from_ints([0, 1, (1 << 511) - 1, 1 << 511, (1 << 1024) - 1], 32)
     assert list(oracle.rsa_hit(oracle.bitlen_rows(G), 1024)) == [False, False, False, True, True]
     assert list(oracle.bitlen_rows(G)) == [0, 1, 511, 512, 1024]
+
+
+def test_cofactors_construction_truth():
+    """N3 factor output (n1 = p * (n1/p)): for every planted hit the
+    oracle's cofactors are the construction's other primes; duplicates give (1, 1)."""
+    ms = synth.moduli(40, 1024, seed=77, n_planted_pairs=2, cliques=(3,), n_duplicates=1)
+    got = oracle.cofactors(ms.N, ms.truth)
+    dup = set(ms.duplicates)
+    for (i, j, g), (ci, cj) in zip(ms.truth, got):
+        if (i, j) in dup:
+            assert (ci, cj) == (1, 1) and g == synth.to_int(ms.N[i])
+        else:
+            assert ci == synth.to_int(ms.P[2 * i + 1]) and cj == synth.to_int(ms.P[2 * j + 1])
+            assert g * ci == synth.to_int(ms.N[i]) and g * cj == synth.to_int(ms.N[j])
+    with pytest.raises(ValueError):
+        oracle.cofactors(ms.N, [(0, 1, 3)])
