@@ -53,6 +53,8 @@ WORKLOADS = {
             "(BASELINE.json configs[3])",
     "cfg5": "cfg5: all-pairs 1024-bit RSA moduli, n=65536 (2,147,450,880 pairs), 33 planted shared primes "
             "(BASELINE.json configs[4])",
+    "cfg2": "cfg2: 2^20 independent 1024-bit pair GCDs, exact mode (bulkgcd_pairs; the first 2^20 pairs i<j "
+            "of a 1,449-moduli pool with 2 planted shared primes; BASELINE.json configs[1])",
 }
 UNIT = "GCD/s"
 OPS_PER_LIMB, OPS_PER_ITER = 4, 16  # SURVEY.md §8(d) M2; DESIGN.md §Roofline
@@ -239,6 +241,150 @@ def run_reference(args):
     print(json.dumps(line))
 
 
+def run_pairs(args):
+    """cfg2 (BASELINE.json configs[1]): bulk execution of 2^20 independent exact
+    GCDs through bulkgcd_pairs.  One step = word-interleave A and B (H1), the
+    pairs kernel (exact mode, L41 + L107 to Y = 0) and the de-interleave of G.
+    N > 1: contiguous chunks of the pairs per rank, no data-path collective
+    ("replicas only" shape); total work fixed -> strong."""
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    import paper_conf_ipps_fujitani15_b200 as bg
+
+    rank, world, local = _env_rank()
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world} (launch N>1 with torchrun)")
+    local = local % torch.cuda.device_count()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("gloo" if BACKEND == "gloo" else "nccl",
+                                **({} if BACKEND == "gloo" else {"device_id": dev}))
+    bg.bulkgcd_device_check()
+    bits, W = 1024, 32
+    A, B, pool = synth.config2()
+    m_all = A.shape[0]
+    lo, hi = m_all * rank // world, m_all * (rank + 1) // world
+    A, B = np.ascontiguousarray(A[lo:hi]), np.ascontiguousarray(B[lo:hi])
+    m = A.shape[0]
+    m_pad = (m + 31) // 32 * 32
+    dA = torch.from_numpy(A.view(np.int32)).to(dev)
+    dB = torch.from_numpy(B.view(np.int32)).to(dev)
+    dAc = torch.empty(m_pad * W, dtype=torch.int32, device=dev)
+    dBc = torch.empty(m_pad * W, dtype=torch.int32, device=dev)
+    dGc = torch.empty(m_pad * W, dtype=torch.int32, device=dev)
+    dG = torch.empty(m * W, dtype=torch.int32, device=dev)
+    dS = torch.zeros(8, dtype=torch.int64, device=dev)
+    k0 = torch.cuda.Event(enable_timing=True)
+    k1 = torch.cuda.Event(enable_timing=True)
+
+    def step(flags=0):
+        bg.bulkgcd_interleave(dA, dAc, m, m_pad, bits, True)
+        bg.bulkgcd_interleave(dB, dBc, m, m_pad, bits, True)
+        k0.record()
+        bg.bulkgcd_pairs_device(dAc, dBc, dGc, m, m_pad, bits, bg.MODE_EXACT, None, dS, flags)
+        k1.record()
+        bg.bulkgcd_interleave(dGc, dG, m, m_pad, bits, False)
+
+    step(bg.FLAG_STATS)  # algorithmic work (untimed stats pass)
+    torch.cuda.synchronize()
+    ctr = dS.cpu().numpy().astype(np.int64)
+    iters, limbs = int(ctr[2]), int(ctr[4])
+    ops_alg = OPS_PER_LIMB * limbs + OPS_PER_ITER * iters
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms, kern_ms = [], []
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record()
+            step()
+            e1.record()
+            e1.synchronize()
+            step_ms.append(e0.elapsed_time(e1))
+            kern_ms.append(k0.elapsed_time(k1))
+    # correctness (outside the timed region): a seeded sample + the planted pairs vs the oracle
+    import oracle
+    G = dG.cpu().numpy().view(np.uint32).reshape(m, W)
+    rng = np.random.default_rng(5)
+    idx = np.unique(rng.integers(0, m, size=min(m, 2048)))
+    ok = bool(np.array_equal(G[idx], oracle.gcd_batch(A[idx], B[idx])))
+    tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        _coll(dist.all_reduce, tot, op=dist.ReduceOp.MAX)
+    step_total_ms, kern_total_ms = float(tot[0]), float(tot[1])
+    # e2e: bulkgcd_pairs with host buffers (H2D of A, B; D2H of G inside the call)
+    e2e = []
+    for _ in range(args.e2e_steps):
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        bg.bulkgcd_pairs(A, B, bits)
+        e2e.append(time.perf_counter() - t0)
+    e2e_t = torch.tensor([sum(e2e)], dtype=torch.float64, device=dev)
+    if world > 1:
+        _coll(dist.all_reduce, e2e_t, op=dist.ReduceOp.MAX)
+    if rank == 0:
+        value = m_all / (step_total_ms / 1e3 / args.steps)
+        peaks, src = _peaks()
+        f_mhz = float(peaks.get("sm_max_mhz", 1965.0))
+        sms = torch.cuda.get_device_properties(dev).multi_processor_count
+        ipc = _int_issue_peak() or 4.0
+        peak_ops = sms * 32 * ipc * f_mhz * 1e6
+        kern_s = kern_total_ms / 1e3 / args.steps
+        achieved = ops_alg / kern_s
+        line = {
+            "metric": "1024-bit GCDs/sec (bulk pairs, exact)", "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_total_ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": WORKLOADS["cfg2"], "pairs": m_all, "bits": bits, "mode": "exact",
+                       "parallelism": f"contiguous chunks x{world} (no collective)",
+                       "l2": "inputs larger than L2 (2 x 128 MiB operands + 128 MiB result)",
+                       "ns_per_gcd": step_total_ms / args.steps * 1e6 / m_all,
+                       "iterations_per_gcd": iters / m, "limb_steps_per_gcd": limbs / m,
+                       "sample_ok": ok, "sample_checked": int(idx.size)},
+            "roofline": {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
+                         "unit": "T int lane-ops/s", "frac": achieved / peak_ops, "traffic": None,
+                         "kernel": f"pairs_kernel<{W}, exact>", "kernel_ms": kern_s * 1e3,
+                         "kernel_share_of_step": kern_total_ms / step_total_ms, "ops_per_gcd": ops_alg / m,
+                         "hbm_bytes_per_gcd_alg": 3 * W * 4,
+                         "hbm_GBps_alg": 3 * W * 4 * m / kern_s / 1e9},
+            "e2e": {"value": m_all / (float(e2e_t[0]) / args.e2e_steps), "unit": UNIT,
+                    "h2d_bytes_per_step": int(A.nbytes + B.nbytes) * world, "d2h_bytes_per_step": int(A.nbytes) * world},
+            "gpu_launches": 4 * args.steps,
+            "clocks": clk.summary(),
+        }
+        if world == 1 and not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline_pairs(A, B)
+        print(json.dumps(line))
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def cpu_baseline_pairs(A, B, target_s: float = 10.0):
+    """The oracle (exact classical Euclid) on a bounded prefix of the cfg2 pairs, all host cores."""
+    import oracle
+    cores = os.cpu_count() or 1
+    k = 1 << 12
+    t0 = time.perf_counter()
+    oracle.gcd_batch(A[:k], B[:k], nthreads=cores)
+    rate = k / (time.perf_counter() - t0)
+    k = int(min(A.shape[0], max(1 << 14, rate * target_s)))
+    t0 = time.perf_counter()
+    oracle.gcd_batch(A[:k], B[:k], nthreads=cores)
+    dt = time.perf_counter() - t0
+    return {"value": k / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"the first {k} of the 2^20 cfg2 pairs, exact classical Euclid (Knuth D), {dt:.1f}s on "
+                      f"{cores} threads"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -253,6 +399,8 @@ def main():
         return run_reference(args)
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
+    if args.workload == "cfg2":
+        return run_pairs(args)
 
     import torch
     import torch.distributed as dist

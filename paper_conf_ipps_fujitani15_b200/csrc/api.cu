@@ -93,7 +93,7 @@ int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m,
     CK(cudaMemsetAsync(scratch, 0, 8 * sizeof(unsigned long long), st));
     PairsArgs a{dA, dB, dG, m, m_pad, scratch + 1, d_iters, scratch + 2, W * 16};
     uint64_t cohorts = (m + 31) / 32;
-    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (cohorts + 3) / 4);
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (cohorts + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
     if (grid == 0) return 0;
     bool stats = (flags & BULKGCD_FLAG_STATS) || d_iters;
     if (mode == BULKGCD_MODE_RSA) {
@@ -114,7 +114,7 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if (c1 <= c0) return 0;
     AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
     uint64_t warps = c1 - c0;
-    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + 3) / 4);
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
     constexpr size_t smem = allpairs_smem_bytes<W>();
     static bool attr_done[2] = {false, false};  // idempotent, benign race
     if (!attr_done[0]) {

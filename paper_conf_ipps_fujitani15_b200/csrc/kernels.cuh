@@ -8,15 +8,33 @@
 
 namespace bulkgcd {
 
-constexpr int THREADS = 128;  // 4 warps per CTA
-#ifndef MIN_BLOCKS
-#define MIN_BLOCKS 3  // CTAs per SM for W <= 32 (3 -> <= 168 registers per thread, no spills)
+#ifndef BULKGCD_THREADS
+#define BULKGCD_THREADS 128  // 4 warps per CTA
+#endif
+constexpr int THREADS = BULKGCD_THREADS;
+constexpr int WARPS_PER_CTA = THREADS / 32;
+#ifndef MIN_WARPS
+// resident warps per SM for W <= 32: 16 -> <= 128 registers per thread.  The hot
+// loop stays spill-free (ptxas spills only cold-section state); 16 warps hide the
+// fixed-latency dependency chains better than 12 (cfg3 292 -> 266 ms).
+#define MIN_WARPS 16
+#endif
+#ifndef MIN_WARPS_W64
+#define MIN_WARPS_W64 8
 #endif
 // CTAs per SM by width: the operands take 2W registers per thread; W = 64
-// (2048-bit) needs ~200 registers, i.e. 2 CTAs (8 warps) per SM.
+// (2048-bit) needs ~200+ registers, i.e. 8 warps per SM.
+// Register cap: __launch_bounds__(THREADS, blocks) by default; -DBULKGCD_MAXNREG=N
+// instead caps every kernel at N registers per thread (__maxnreg__).
+#ifdef BULKGCD_MAXNREG
+#define BULKGCD_BOUNDS(W) __maxnreg__(BULKGCD_MAXNREG)
+#else
+#define BULKGCD_BOUNDS(W) __launch_bounds__(THREADS, Occ<W>::blocks)
+#endif
 template <int W>
 struct Occ {
-    static constexpr int blocks = W >= 64 ? 2 : MIN_BLOCKS;
+    static constexpr int warps = W >= 64 ? MIN_WARPS_W64 : MIN_WARPS;
+    static constexpr int blocks = warps / WARPS_PER_CTA > 0 ? warps / WARPS_PER_CTA : 1;
 };
 
 // ------------------------------------------------------------------ layouts
@@ -179,7 +197,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
         bool fin = live & !run & !bad;
-        bool need = sink.quick(fin, lY, tY, lX, tX) | bad;
+        bool need = sink.quick_hot(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
         unsigned bneed = __ballot_sync(FULL, need), btop = __ballot_sync(FULL, top);
         if (bneed != 0u) {
@@ -375,6 +393,9 @@ struct PairsSinkExact {
         }
         return fin && lY == 0;
     }
+    __device__ __forceinline__ bool quick_hot(bool fin, int lX, uint64_t tX, int lY, uint64_t tY) {
+        return quick(fin, lX, tX, lY, tY);
+    }
     // Y = 0: g = X (possibly long), written with the common power of two restored
     __device__ __forceinline__ void cold(bool need, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX, int lY,
                                          uint64_t tY, int s) {
@@ -391,6 +412,7 @@ struct PairsSinkRsa {
     uint32_t *G;
     uint64_t i, stride;
     __device__ __forceinline__ bool quick(bool fin, int, uint64_t, int, uint64_t) { return fin; }
+    __device__ __forceinline__ bool quick_hot(bool fin, int, uint64_t, int, uint64_t) { return fin; }
     __device__ __forceinline__ void cold(bool need, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX, int lY,
                                          uint64_t tY, int s) {
         if (!need) return;
@@ -406,7 +428,7 @@ struct PairsSinkRsa {
 };
 
 template <int W, bool RSA, bool STATS>
-__global__ void __launch_bounds__(THREADS, Occ<W>::blocks) pairs_kernel(PairsArgs a) {
+__global__ void BULKGCD_BOUNDS(W) pairs_kernel(PairsArgs a) {
     const int lane = threadIdx.x & 31;
     uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0, passw = 0;
     for (;;) {
@@ -517,6 +539,9 @@ struct HitSink {
     uint32_t i, j;
     // a lane that stops with Y != 0 is coprime-mode ("return 1", L243/L251): nothing to report
     __device__ __forceinline__ bool quick(bool fin, int, uint64_t, int lY, uint64_t) { return fin && lY == 0; }
+    // In the hot loop a lane only finishes with Y = X' != 0 (a zero X' sets `post` and goes cold):
+    // it is coprime-mode, nothing to report.
+    __device__ __forceinline__ bool quick_hot(bool, int, uint64_t, int, uint64_t) { return false; }
     // Compacting hit writer: warp ballot + one atomic per warp (north_star (4)).
     __device__ __forceinline__ void cold(bool hit, uint32_t (&X)[W], uint32_t (&Y)[W], int lX, uint64_t tX, int lY,
                                          uint64_t tY, int s) {
@@ -608,7 +633,7 @@ __device__ __forceinline__ void cohort_coords(uint64_t c, uint64_t n, uint64_t &
 }
 
 template <int W, bool STATS>
-__global__ void __launch_bounds__(THREADS, Occ<W>::blocks) allpairs_kernel(AllPairsArgs a) {
+__global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     StageBuf<W> *buf = reinterpret_cast<StageBuf<W> *>(smem_raw) + 2 * warp;
