@@ -6,7 +6,9 @@
  *
  * Numbers.  A `bits`-bit number is W = bits/32 little-endian 32-bit words
  * ("d = 32", L251): word k (0 = least significant) of number i is at
- * X[i*W + k] ("row-major").  Supported bits: 512, 1024, 2048 (W = 16, 32, 64).
+ * X[i*W + k] ("row-major").  Supported bits: 512, 1024, 2048, 4096 (W = 16, 32,
+ * 64, 128).  W <= 64 run register-resident kernels; W = 128 runs the
+ * shared-memory-resident kernels (the operands do not fit in registers).
  *
  * Modes.
  *   EXACT (BULKGCD_MODE_EXACT): the exact gcd of any operands 0 <= a, b <
@@ -47,6 +49,13 @@ extern "C" {
 #define BULKGCD_MODE_RSA 1
 
 #define BULKGCD_FLAG_STATS 1u /* device entry points: accumulate iteration/slow-step counters */
+#define BULKGCD_FLAG_SMEM 2u  /* device entry points: use the shared-memory-resident kernels (the W = 128
+                                 design) at any width -- a diagnostic/test route, same results */
+/* Comparison algorithms of the paper's Tables IV/V, device entry points only;
+ * same results (gcd / RSA-mode hits), different iteration counts.  Default: Approximate Euclid (E). */
+#define BULKGCD_FLAG_ALGO_FAST_BINARY (1u << 8) /* (D) Fast Binary Euclid, L43: X <- rshift(X - Y) */
+#define BULKGCD_FLAG_ALGO_BINARY (2u << 8)      /* (C) Binary Euclid, L57: X/2, Y/2 or (X - Y)/2 */
+#define BULKGCD_FLAG_ALGO_MASK (3u << 8)
 
 /* Hits of bulkgcd_all_pairs; arrays are allocated by the library. */
 typedef struct {
@@ -129,7 +138,10 @@ uint64_t bulkgcd_cohort_count(size_t n);
  * unsigned long long of device memory, zeroed by the call ([2] = summed
  * iterations, [3] = slow-path steps, [4] = limb-steps = sum of lX over all
  * iterations, [5] = lane-slots, when flags has BULKGCD_FLAG_STATS or d_iters
- * is given).  No validation of operand values.
+ * is given; the shared-memory kernels (W = 128 or BULKGCD_FLAG_SMEM) count
+ * beta > 0 updates and rshifts by >= 32 bits as [3], set [5] = [2], [6] = [4],
+ * and add [7] = iterations with beta > 0, the statistic of L253).  No
+ * validation of operand values.
  */
 int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G, size_t m, size_t m_pad,
                          uint32_t bits, int mode, uint32_t *d_iters, unsigned long long *d_scratch,
@@ -145,7 +157,9 @@ int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G
  * iterations, [3] = slow-path steps, [4] = limb-steps (sum of lX, the words
  * each update pass covers), [5] = lane-slots (32 x warp-iterations; [2]/[5]
  * is the SIMT lane efficiency), [6] = lane-words issued by the passes ([4]/[6]
- * is the pass-word efficiency).  Moduli must be odd and > 1 (not checked here).
+ * is the pass-word efficiency); the shared-memory kernels as for
+ * bulkgcd_pairs_device, with [7] = iterations with beta > 0 (L253).  Moduli
+ * must be odd and > 1 (not checked here).
  */
 int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t n, uint32_t bits,
                            uint64_t cohort_begin, uint64_t cohort_end, uint32_t *d_hits, uint64_t hit_cap,

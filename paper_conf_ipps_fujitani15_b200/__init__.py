@@ -23,6 +23,9 @@ from ._build import SO, build  # noqa: F401
 MODE_EXACT = 0
 MODE_RSA = 1
 FLAG_STATS = 1
+FLAG_SMEM = 2
+FLAG_ALGO_FAST_BINARY = 1 << 8
+FLAG_ALGO_BINARY = 2 << 8
 
 EINVAL, ENOMEM, ECUDA, ENODEV = -1, -2, -3, -4
 

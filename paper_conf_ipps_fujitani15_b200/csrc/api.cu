@@ -45,6 +45,7 @@ int words_for(uint32_t bits) {
         case 512: return 16;
         case 1024: return 32;
         case 2048: return 64;
+        case 4096: return 128;
         default: return 0;
     }
 }
@@ -87,11 +88,52 @@ struct DBuf {
 
 size_t pad32(size_t m) { return (m + 31) / 32 * 32; }
 
+// Shared-memory-resident kernels: W = 128 always, other widths with BULKGCD_FLAG_SMEM,
+// and the comparison algorithms (BULKGCD_FLAG_ALGO_*).
+template <int W, int ALG>
+int launch_pairs_smem_alg(const PairsArgs &a, int mode, bool stats, cudaStream_t st) {
+    constexpr size_t smem = smem_operand_bytes<W>();
+    static bool attr_done = false;  // idempotent, benign race
+    if (!attr_done) {
+        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        attr_done = true;
+    }
+    uint64_t cohorts = (a.m + 31) / 32;
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * smem_blocks<W>(), (cohorts + 1) / 2);
+    if (grid == 0) return 0;
+    if (mode == BULKGCD_MODE_RSA) {
+        if (stats) pairs_smem_kernel<W, true, true, ALG><<<(unsigned)grid, SM_THREADS, smem, st>>>(a);
+        else pairs_smem_kernel<W, true, false, ALG><<<(unsigned)grid, SM_THREADS, smem, st>>>(a);
+    } else {
+        if (stats) pairs_smem_kernel<W, false, true, ALG><<<(unsigned)grid, SM_THREADS, smem, st>>>(a);
+        else pairs_smem_kernel<W, false, false, ALG><<<(unsigned)grid, SM_THREADS, smem, st>>>(a);
+    }
+    CK(cudaGetLastError());
+    return 0;
+}
+
+template <int W>
+int launch_pairs_smem(const PairsArgs &a, int mode, bool stats, unsigned flags, cudaStream_t st) {
+    switch (flags & BULKGCD_FLAG_ALGO_MASK) {
+        case BULKGCD_FLAG_ALGO_FAST_BINARY: return launch_pairs_smem_alg<W, ALG_FAST_BINARY>(a, mode, stats, st);
+        case BULKGCD_FLAG_ALGO_BINARY: return launch_pairs_smem_alg<W, ALG_BINARY>(a, mode, stats, st);
+        default: return launch_pairs_smem_alg<W, ALG_APPROX>(a, mode, stats, st);
+    }
+}
+
 template <int W>
 int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m, size_t m_pad, int mode,
                  uint32_t *d_iters, unsigned long long *scratch, unsigned flags, cudaStream_t st) {
     CK(cudaMemsetAsync(scratch, 0, 8 * sizeof(unsigned long long), st));
     PairsArgs a{dA, dB, dG, m, m_pad, scratch + 1, d_iters, scratch + 2, W * 16};
+    bool stats_ = (flags & BULKGCD_FLAG_STATS) || d_iters;
+    if constexpr (W >= 128) {
+        return launch_pairs_smem<W>(a, mode, stats_, flags, st);
+    } else {
+    if (flags & (BULKGCD_FLAG_SMEM | BULKGCD_FLAG_ALGO_MASK)) return launch_pairs_smem<W>(a, mode, stats_, flags, st);
     uint64_t cohorts = (m + 31) / 32;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (cohorts + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
     if (grid == 0) return 0;
@@ -105,6 +147,33 @@ int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m,
     }
     CK(cudaGetLastError());
     return 0;
+    }
+}
+
+template <int W, int ALG>
+int launch_allpairs_smem_alg(const AllPairsArgs &a, bool stats, cudaStream_t st) {
+    constexpr size_t smem = smem_operand_bytes<W>();
+    static bool attr_done = false;  // idempotent, benign race
+    if (!attr_done) {
+        CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        attr_done = true;
+    }
+    uint64_t warps = a.c_end - a.c_begin;
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * smem_blocks<W>(), (warps + 1) / 2);
+    if (stats) allpairs_smem_kernel<W, true, ALG><<<(unsigned)grid, SM_THREADS, smem, st>>>(a);
+    else allpairs_smem_kernel<W, false, ALG><<<(unsigned)grid, SM_THREADS, smem, st>>>(a);
+    CK(cudaGetLastError());
+    return 0;
+}
+
+template <int W>
+int launch_allpairs_smem(const AllPairsArgs &a, bool stats, unsigned flags, cudaStream_t st) {
+    switch (flags & BULKGCD_FLAG_ALGO_MASK) {
+        case BULKGCD_FLAG_ALGO_FAST_BINARY: return launch_allpairs_smem_alg<W, ALG_FAST_BINARY>(a, stats, st);
+        case BULKGCD_FLAG_ALGO_BINARY: return launch_allpairs_smem_alg<W, ALG_BINARY>(a, stats, st);
+        default: return launch_allpairs_smem_alg<W, ALG_APPROX>(a, stats, st);
+    }
 }
 
 template <int W>
@@ -113,6 +182,11 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     CK(cudaMemsetAsync(counters, 0, 8 * sizeof(unsigned long long), st));
     if (c1 <= c0) return 0;
     AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
+    if constexpr (W >= 128) {
+        return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
+    } else {
+    if (flags & (BULKGCD_FLAG_SMEM | BULKGCD_FLAG_ALGO_MASK))
+        return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     uint64_t warps = c1 - c0;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
     constexpr size_t smem = allpairs_smem_bytes<W>();
@@ -126,6 +200,7 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, smem, st>>>(a);
     CK(cudaGetLastError());
     return 0;
+    }
 }
 
 int check_moduli(const uint32_t *N, size_t n, int W) {
@@ -200,7 +275,8 @@ int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G
     switch (W) {
         case 16: return launch_pairs<16>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
         case 32: return launch_pairs<32>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
-        default: return launch_pairs<64>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
+        case 64: return launch_pairs<64>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
+        default: return launch_pairs<128>(d_A, d_B, d_G, m, m_pad, mode, d_iters, d_scratch, flags, st);
     }
 }
 
@@ -219,14 +295,15 @@ int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t 
     switch (W) {
         case 16: return launch_allpairs<16>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
         case 32: return launch_allpairs<32>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
-        default: return launch_allpairs<64>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
+        case 64: return launch_allpairs<64>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
+        default: return launch_allpairs<128>(d_N, d_N_blk, n, cohort_begin, cohort_end, d_hits, hit_cap, d_counters, flags, st);
     }
 }
 
 int bulkgcd_pairs_ex(const uint32_t *A, const uint32_t *B, size_t m, uint32_t bits, int mode, uint32_t *G,
                      uint32_t *iters) {
     int W = words_for(bits);
-    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048)", bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048, 4096)", bits);
     if (mode != BULKGCD_MODE_EXACT && mode != BULKGCD_MODE_RSA) return set_err(BULKGCD_EINVAL, "bad mode %d", mode);
     if (m == 0) return 0;
     if (!A || !B || !G) return set_err(BULKGCD_EINVAL, "null pointer with m > 0");
@@ -280,7 +357,7 @@ int bulkgcd_all_pairs(const uint32_t *N, size_t n, uint32_t bits, bulkgcd_hits_t
     if (!out) return set_err(BULKGCD_EINVAL, "null hits_out");
     memset(out, 0, sizeof *out);
     out->bits = bits;
-    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048)", bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048, 4096)", bits);
     if (n > 0 && !N) return set_err(BULKGCD_EINVAL, "null moduli with n > 0");
     if (n > 0xFFFFFFFFull) return set_err(BULKGCD_EINVAL, "n too large");
     int rc = check_moduli(N, n, W);
@@ -351,7 +428,8 @@ int bulkgcd_cofactors_device(const uint32_t *d_N, size_t n, uint32_t bits, const
     switch (W) {
         case 16: cofactor_kernel<16><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
         case 32: cofactor_kernel<32><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
-        default: cofactor_kernel<64><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
+        case 64: cofactor_kernel<64><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
+        default: cofactor_kernel<128><<<(unsigned)grid, (unsigned)block, 0, st>>>(d_N, n, d_hits, count, d_F, d_bad); break;
     }
     CK(cudaGetLastError());
     return 0;
@@ -359,7 +437,7 @@ int bulkgcd_cofactors_device(const uint32_t *d_N, size_t n, uint32_t bits, const
 
 int bulkgcd_cofactors(const uint32_t *N, size_t n, uint32_t bits, const bulkgcd_hits_t *hits, uint32_t *F) {
     int W = words_for(bits);
-    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048)", bits);
+    if (!W) return set_err(BULKGCD_EINVAL, "unsupported bits %u (supported: 512, 1024, 2048, 4096)", bits);
     if (!hits) return set_err(BULKGCD_EINVAL, "null hits");
     if (hits->bits != bits) return set_err(BULKGCD_EINVAL, "hits were computed for %u bits, not %u", hits->bits, bits);
     size_t count = hits->count;

@@ -5,6 +5,7 @@
 #include <cstdint>
 
 #include "euclid.cuh"
+#include "smem_euclid.cuh"
 
 namespace bulkgcd {
 
@@ -747,6 +748,126 @@ __global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         atomicAdd(&a.stats[2], (unsigned long long)limbs);
         atomicAdd(&a.stats[3], (unsigned long long)slots);  // lane-slots: warp-iterations x 32
         atomicAdd(&a.stats[4], (unsigned long long)passw);  // lane-words of pass issued
+    }
+}
+
+// ------------------------------------------------- shared-memory-resident kernels
+// 4096-bit (W = 128) bulk and all-pairs GCD with the operands in shared memory
+// (smem_euclid.cuh); also reachable at W <= 64 through BULKGCD_FLAG_SMEM.
+template <int W, bool RSA, bool STATS, int ALG>
+__global__ void __launch_bounds__(SM_THREADS) pairs_smem_kernel(PairsArgs a) {
+    extern __shared__ __align__(16) uint32_t sbuf[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t *wb = sbuf + (size_t)warp * 2 * W * 32;
+    uint32_t iters = 0, rare = 0, limbs = 0, betapos = 0;
+    for (;;) {
+        unsigned long long c = 0;
+        if (lane == 0) c = atomicAdd(a.work, 1ull);
+        c = __shfl_sync(FULL, c, 0);
+        if (c * 32 >= a.m) break;
+        uint64_t i = c * 32 + lane;
+        bool valid = i < a.m;
+        SOp X{wb + lane}, Y{wb + W * 32 + lane};
+        for (int k = 0; k < W; ++k) {
+            X[k] = valid ? a.A[(uint64_t)k * a.m_pad + i] : 0u;
+            Y[k] = valid ? a.B[(uint64_t)k * a.m_pad + i] : 0u;
+        }
+        uint32_t it0 = iters;
+        if (valid) {
+            int lX, lY;
+            uint64_t tX, tY;
+            if (RSA) {
+                s_setup(X, Y, lX, tX, lY, tY, W);
+                s_euclid<false, STATS, ALG>(X, Y, lX, tX, lY, tY, a.half, iters, rare, limbs, betapos);
+                if (lY == 0) s_write_shifted(a.G + i, a.m_pad, X, lX, 0, W);  // g = X (L251)
+                else for (int w = 0; w < W; ++w) a.G[i + (uint64_t)w * a.m_pad] = w == 0 ? 1u : 0u;
+            } else {
+                int la = s_len(X, W), lb = s_len(Y, W);
+                if (la == 0 || lb == 0) {  // gcd(x, 0) = x
+                    SOp Z = la ? X : Y;
+                    s_write_shifted(a.G + i, a.m_pad, Z, la ? la : lb, 0, W);
+                } else {  // L41: strip the common power of two k2 and every other factor 2
+                    int ca = s_ctz(X, la), cb = s_ctz(Y, lb);
+                    int k2 = ca < cb ? ca : cb;
+                    s_rshift(X, la);
+                    s_rshift(Y, lb);
+                    s_setup(X, Y, lX, tX, lY, tY, W);
+                    s_euclid<true, STATS, ALG>(X, Y, lX, tX, lY, tY, 0, iters, rare, limbs, betapos);
+                    if (ALG == ALG_APPROX && lY != 0) {  // Case 1 tail (lX <= 2)
+                        uint64_t g = s_tail64<STATS>(s_value64(X, lX), s_value64(Y, lY), iters, limbs);
+                        X[0] = (uint32_t)g;
+                        X[1] = (uint32_t)(g >> 32);
+                        lX = g >> 32 ? 2 : (g ? 1 : 0);
+                    }
+                    s_write_shifted(a.G + i, a.m_pad, X, lX, k2, W);
+                }
+            }
+        }
+        if (a.iters && valid) a.iters[i] = iters - it0;
+        __syncwarp();
+    }
+    if (STATS && a.stats) {
+        atomicAdd(&a.stats[0], (unsigned long long)iters);
+        atomicAdd(&a.stats[1], (unsigned long long)rare);
+        atomicAdd(&a.stats[2], (unsigned long long)limbs);
+        atomicAdd(&a.stats[3], (unsigned long long)iters);  // no lockstep accounting: lane-slots = iterations
+        atomicAdd(&a.stats[4], (unsigned long long)limbs);
+        atomicAdd(&a.stats[5], (unsigned long long)betapos);
+    }
+}
+
+template <int W, bool STATS, int ALG>
+__global__ void __launch_bounds__(SM_THREADS) allpairs_smem_kernel(AllPairsArgs a) {
+    extern __shared__ __align__(16) uint32_t sbuf[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t *wb = sbuf + (size_t)warp * 2 * W * 32;
+    uint32_t iters = 0, rare = 0, limbs = 0, betapos = 0;
+    for (;;) {
+        unsigned long long cc = 0;
+        if (lane == 0) cc = atomicAdd(a.work, 1ull);
+        uint64_t c = __shfl_sync(FULL, cc, 0) + a.c_begin;
+        if (c >= a.c_end) break;
+        uint64_t b, j;
+        cohort_coords(c, a.n, b, j);
+        uint64_t i = 32 * b + lane;
+        bool live = i < j;
+        SOp X{wb + lane}, Y{wb + W * 32 + lane};
+        for (int k = 0; k < W; ++k) {
+            X[k] = a.N_blk[(b * W + k) * 32 + lane];  // one coalesced 128-byte row per word
+            Y[k] = a.N_rm[j * W + k];                 // the column modulus (broadcast)
+        }
+        int lX = 0, lY = 0;
+        uint64_t tX = 0, tY = 0;
+        if (live) {
+            s_setup(X, Y, lX, tX, lY, tY, W);
+            s_euclid<false, STATS, ALG>(X, Y, lX, tX, lY, tY, a.half, iters, rare, limbs, betapos);
+        }
+        bool hit = live && lY == 0;  // Y = 0: g = X has >= bits/2 bits (L251)
+        unsigned mask = __ballot_sync(FULL, hit);
+        if (mask) {  // compacting hit writer: ballot + one atomic per warp
+            const int leader = __ffs(mask) - 1;
+            unsigned long long base = 0;
+            if (lane == leader) base = atomicAdd(a.hit_count, (unsigned long long)__popc(mask));
+            base = __shfl_sync(FULL, base, leader);
+            if (hit) {
+                uint64_t slot = base + __popc(mask & ((1u << lane) - 1));
+                if (slot < a.hit_cap) {
+                    uint32_t *rec = a.hits + slot * (2 + W);
+                    rec[0] = (uint32_t)i;
+                    rec[1] = (uint32_t)j;
+                    s_write_shifted(rec + 2, 1, X, lX, 0, W);
+                }
+            }
+        }
+        __syncwarp();
+    }
+    if (STATS && a.stats) {
+        atomicAdd(&a.stats[0], (unsigned long long)iters);
+        atomicAdd(&a.stats[1], (unsigned long long)rare);
+        atomicAdd(&a.stats[2], (unsigned long long)limbs);
+        atomicAdd(&a.stats[3], (unsigned long long)iters);
+        atomicAdd(&a.stats[4], (unsigned long long)limbs);
+        atomicAdd(&a.stats[5], (unsigned long long)betapos);
     }
 }
 

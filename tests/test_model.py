@@ -136,3 +136,32 @@ def test_table4_means(bits, npairs):
     paper_a = tab[("nonterm", bits)][0]
     se = math.sqrt(orig.var() / orig.size + orig.var() / 10000)
     assert abs(orig.mean() - paper_a) <= 3 * se + 0.05, (bits, orig.mean(), paper_a)
+
+
+def test_table1_binary_and_fast_binary():
+    """Table I (L47, L69-L81): on X = 1043915, Y = 768955 the Binary Euclidean
+    algorithm takes 24 iterations and Fast Binary 16; both return 5."""
+    for fn, it in ((am.binary_euclid, 24), (am.fast_binary_euclid, 16)):
+        t = fn(1043915, 768955)
+        assert (t.gcd, t.iterations) == (5, it)
+        assert fn(768955, 1043915).iterations == it  # X < Y on entry: swap first
+
+
+@pytest.mark.parametrize("bits,npairs", [(512, 1500), (1024, 800)])
+def test_table4_binary_columns(bits, npairs):
+    """Table IV columns (C) Binary and (D) Fast Binary, both modes, within 3 combined
+    standard errors of the paper's 10,000-pair means (comparison algorithms, N2)."""
+    tab = _table4()
+    ms = synth.moduli(npairs + 1, bits, seed=4000 + bits)
+    N = synth.ints(ms.N)
+    for col, fn in ((2, am.binary_euclid), (3, am.fast_binary_euclid)):
+        for mode, early in (("early", bits), ("nonterm", None)):
+            arr = np.array([fn(N[k], N[k + 1], early).iterations for k in range(npairs)], float)
+            paper = tab[(mode, bits)][col]
+            se = math.sqrt(arr.var() / arr.size + arr.var() / 10000)
+            # (C) early-terminate: the paper gives no listing, only (E)'s (L255); with (E)'s loop-head
+            # test our mean is 0.2-0.5% below the printed one (DESIGN.md reading 20): checked to 0.6%.
+            tol = 0.006 * paper if (col, mode) == (2, "early") else 3 * se + 0.05
+            assert abs(arr.mean() - paper) <= tol, (col, mode, bits, arr.mean(), paper, se)
+    g = [am.binary_euclid(N[k], N[k + 1]).gcd for k in range(50)]
+    assert g == [math.gcd(N[k], N[k + 1]) for k in range(50)]
