@@ -394,6 +394,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--workload", default="cfg3", choices=sorted(WORKLOADS))
+    ap.add_argument("--algo", default="E", choices=["E", "D", "C"],
+                    help="all-pairs ablation (SURVEY.md §8(f) N2): E = Approximate Euclid (the product), "
+                         "D = Fast Binary, C = Binary Euclid (the paper's Table V columns)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -448,10 +451,12 @@ def main():
     gbuf = torch.empty(world * cap * (2 + W), dtype=torch.int32, device=dev)
     gcnt = torch.empty(world, dtype=torch.int64, device=dev)
 
+    algo_flag = {"E": 0, "D": bg.FLAG_ALGO_FAST_BINARY, "C": bg.FLAG_ALGO_BINARY}[args.algo]
+
     def step():
         runner.layout()
         k0.record()
-        runner.search()
+        runner.search(algo_flag)
         k1.record()
         if world > 1:
             # the exchange step: NCCL all-gather of the hit counts and fixed-capacity hit buffers
@@ -460,7 +465,7 @@ def main():
 
     # ---- algorithmic work of one launch (stats pass, untimed)
     runner.layout()
-    runner.search(bg.FLAG_STATS)
+    runner.search(bg.FLAG_STATS | algo_flag)
     torch.cuda.synchronize()
     ctr = runner.d_ctr.cpu().numpy().astype(np.int64)
     iters, limbs = int(ctr[2]), int(ctr[4])
@@ -518,6 +523,8 @@ def main():
     e2e_ms = []
     Nh = np.ascontiguousarray(N)
     d2h = 0
+    if args.algo != "E":
+        args.e2e_steps = 0  # the public API runs (E); an ablation has no end-to-end line
     for _ in range(args.e2e_steps):
         flush.fill_(3)
         torch.cuda.synchronize()
@@ -534,7 +541,7 @@ def main():
     e2e_t = torch.tensor([sum(e2e_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         _coll(dist.all_reduce, e2e_t, op=dist.ReduceOp.MAX)
-    e2e_value = pairs / (float(e2e_t[0]) / 1e3 / args.e2e_steps)
+    e2e_value = pairs / (float(e2e_t[0]) / 1e3 / args.e2e_steps) if args.e2e_steps else None
 
     if rank == 0:
         value = pairs / (step_total_ms / 1e3 / args.steps)
@@ -554,6 +561,9 @@ def main():
             "data": "synthetic",
             "config": {"workload": WORKLOADS[args.workload],
                        "n": n, "bits": bits, "pairs": pairs, "mode": "rsa-early-terminate",
+                       "algorithm": {"E": "approximate-euclid (register-resident)",
+                                     "D": "fast-binary-euclid (ablation, " + ("register" if bits == 1024 else "smem") + ")",
+                                     "C": "binary-euclid (ablation, smem)"}[args.algo],
                        "parallelism": f"row-band x{world}" + (" + NCCL hit all-gather" if world > 1 else ""),
                        "l2": "flushed before every step (256 MiB write); inputs 2 MiB",
                        "ns_per_gcd": step_total_ms / args.steps * 1e6 / pairs,
@@ -561,7 +571,8 @@ def main():
                        "hits_ok": bool(ok), "hits": len(found), "wall_s": t_wall},
             "roofline": {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
                          "unit": "T int lane-ops/s", "frac": achieved / peak_ops, "traffic": _traffic(),
-                         "kernel": f"allpairs_kernel<{W}>", "kernel_ms": kern_s * 1e3,
+                         "kernel": f"allpairs_kernel<{W}>" if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
+                         "kernel_ms": kern_s * 1e3,
                          "kernel_share_of_step": kern_total_ms / step_total_ms,
                          "ops_per_gcd": ops_alg / pairs,
                          "peak_source": (f"measured integer issue ceiling {ipc:.3f} warp-instr/clk/SM "
@@ -570,7 +581,7 @@ def main():
                                         f"{sms} SMs x 128 lanes x {f_mhz:.0f} MHz (guide unit counts)",
                          "peak_guide": guide_ops / 1e12, "frac_of_guide_peak": achieved / guide_ops},
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,
-                    "d2h_bytes_per_step": int(d2h) * world},
+                    "d2h_bytes_per_step": int(d2h) * world} if e2e_value else None,
             "gpu_launches": 2 * args.steps,
             "clocks": clk.summary(),
         }

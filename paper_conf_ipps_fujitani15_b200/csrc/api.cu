@@ -185,7 +185,10 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if constexpr (W >= 128) {
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     } else {
-    if (flags & (BULKGCD_FLAG_SMEM | BULKGCD_FLAG_ALGO_MASK))
+    // (D) on the register harness at 1024 bits (the paper's headline width); other algorithm routes: smem
+    constexpr bool reg_fastbin = W == 32;
+    unsigned algo = flags & BULKGCD_FLAG_ALGO_MASK;
+    if ((flags & BULKGCD_FLAG_SMEM) || (algo && !(reg_fastbin && algo == BULKGCD_FLAG_ALGO_FAST_BINARY)))
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     uint64_t warps = c1 - c0;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
@@ -194,7 +197,19 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if (!attr_done[0]) {
         CK(cudaFuncSetAttribute(allpairs_kernel<W, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         CK(cudaFuncSetAttribute(allpairs_kernel<W, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        if constexpr (reg_fastbin) {
+            CK(cudaFuncSetAttribute(allpairs_kernel<W, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(allpairs_kernel<W, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        }
         attr_done[0] = true;
+    }
+    if constexpr (reg_fastbin) {
+        if (algo == BULKGCD_FLAG_ALGO_FAST_BINARY) {
+            if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
+            else allpairs_kernel<W, false, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
+            CK(cudaGetLastError());
+            return 0;
+        }
     }
     if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
     else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, smem, st>>>(a);

@@ -142,7 +142,7 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
 // and returns true if a finished lane needs cold(...) (warp-converged, with
 // the operand registers); scalar-only finishes are handled by quick itself.
-template <int W, bool STATS, bool EXACT, class Cond, class Sink, class Parker>
+template <int W, bool STATS, bool EXACT, class Cond, class Sink, class Parker, bool FASTBIN = false>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, Parker &pk, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
@@ -194,7 +194,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
             }
         }
         bool full, post, lt;
-        hot_iter<W, EXACT>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
+        hot_iter<W, EXACT, FASTBIN>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
         bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
         bool fin = live & !run & !bad;
@@ -633,7 +633,8 @@ __device__ __forceinline__ void cohort_coords(uint64_t c, uint64_t n, uint64_t &
     j = 32 * b + 1 + (c - cohorts_before(b, n));
 }
 
-template <int W, bool STATS>
+// FASTBIN: the Fast Binary Euclid ablation (N2) on the same register-resident harness.
+template <int W, bool STATS, bool FASTBIN = false>
 __global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -691,7 +692,7 @@ __global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         unsigned K = pk.K;
         if (!allow_park) pk.K = 0;
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, pi, pj};
-        euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
+        euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk), FASTBIN>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
                                      slots, passw);
         pk.K = K;
     };
@@ -729,11 +730,11 @@ __global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
         if (ParkCfg<W>::on) {
-            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
+            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk), FASTBIN>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
                                          limbs, slots, passw);
         } else {
             NoPark np;
-            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
+            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, NoPark, FASTBIN>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
                                          limbs, slots, passw);
         }
         slot ^= 1;

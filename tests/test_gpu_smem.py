@@ -155,3 +155,55 @@ def test_smem_flag_matches_register_kernels(bg, bits):
         out.append((sorted((int(r[0]), int(r[1]), synth.to_int(r[2:])) for r in rec), int(c[2]), int(c[4])))
     assert out[0] == out[1]
     assert out[0][0] == ms.truth
+
+
+# ------------------------------------- comparison algorithms (C), (D) (N2)
+@pytest.mark.parametrize("bits", [512, 1024])
+def test_comparison_algorithms_parity(bg, bits):
+    """BULKGCD_FLAG_ALGO_BINARY / _FAST_BINARY: per-pair gcd and iteration count equal
+    the model's Binary (L57) / Fast Binary (L43) Euclid, both modes; gcds equal the oracle."""
+    W = bits // 32
+    ms = synth.moduli(161, bits, seed=bits + 21, n_planted_pairs=4, n_duplicates=1)
+    N = synth.ints(ms.N)
+    A, B = ms.N[:-1], ms.N[1:]
+    ii = list(range(160)) + [a for a, b, _ in ms.truth]
+    jj = list(range(1, 161)) + [b for a, b, _ in ms.truth]
+    A = ms.N[ii]
+    B = ms.N[jj]
+    gx = oracle.gcd_batch(A, B)
+    for flag, fn in ((bg.FLAG_ALGO_BINARY, am.binary_euclid), (bg.FLAG_ALGO_FAST_BINARY, am.fast_binary_euclid)):
+        for mode, early in ((bg.MODE_EXACT, None), (bg.MODE_RSA, bits)):
+            G, it, _ = _pairs_device(bg, A, B, bits, mode, flag)
+            for k in range(len(ii)):
+                t = fn(N[ii[k]], N[jj[k]], early)
+                assert synth.to_int(G[k]) == t.gcd, (flag, mode, k)
+                assert int(it[k]) == t.iterations, (flag, mode, k, int(it[k]), t.iterations)
+            if mode == bg.MODE_EXACT:
+                assert np.array_equal(G, gx)
+    Ae, Be = synth.mixed_pairs(500, bits, seed=bits + 22)  # even / zero / odd mixes, exact mode
+    Ah, Bh = synth.from_ints(Ae, W), synth.from_ints(Be, W)
+    for flag in (bg.FLAG_ALGO_BINARY, bg.FLAG_ALGO_FAST_BINARY):
+        G, _, _ = _pairs_device(bg, Ah, Bh, bits, bg.MODE_EXACT, flag)
+        assert np.array_equal(G, oracle.gcd_batch(Ah, Bh))
+
+
+def test_comparison_algorithms_all_pairs(bg, cfg1):
+    """The all-pairs search gives the same (exact) hit set under (C), (D) and (E)."""
+    dev = torch.device("cuda")
+    W = 32
+    dN = torch.from_numpy(cfg1.N.view(np.int32)).to(dev)
+    dBk = torch.empty(bg.bulkgcd_blocked_words(cfg1.m, 1024), dtype=torch.int32, device=dev)
+    bg.bulkgcd_layout_blocked(dN, dBk, cfg1.m, 1024)
+    iters = {}
+    for name, flag in (("E", 0), ("D", bg.FLAG_ALGO_FAST_BINARY), ("C", bg.FLAG_ALGO_BINARY)):
+        dH = torch.zeros(64 * (2 + W), dtype=torch.int32, device=dev)
+        dC = torch.zeros(8, dtype=torch.int64, device=dev)
+        bg.bulkgcd_all_pairs_band(dN, dBk, cfg1.m, 1024, 0, bg.bulkgcd_cohort_count(cfg1.m), dH, 64, dC,
+                                  flag | bg.FLAG_STATS)
+        torch.cuda.synchronize()
+        c = dC.cpu().numpy()
+        rec = dH.cpu().numpy().view(np.uint32).reshape(-1, 2 + W)[:int(c[0])]
+        assert sorted((int(r[0]), int(r[1]), synth.to_int(r[2:])) for r in rec) == cfg1.truth, name
+        iters[name] = int(c[2])
+    # Table IV's ordering (L249): (E) about half of (D), about a quarter of (C)
+    assert 1.7 < iters["D"] / iters["E"] < 2.2 and 3.4 < iters["C"] / iters["E"] < 4.3, iters
