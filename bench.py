@@ -16,11 +16,13 @@ value   : device-timed (CUDA events, sum over the K steps, max over ranks),
 e2e     : the same metric through the public API with HOST buffers: N = 1:
           bulkgcd_all_pairs() (C ABI: H2D, kernels, D2H, sort); N > 1:
           dist.all_pairs_distributed() per rank.  Host-timed per call.
-roofline: the all-pairs kernel, integer-issue bound ("alu"): algorithmic
-          lane-ops per launch (4 per limb-step + 16 per
-          iteration, counted exactly by the kernel's stats pass on the same
-          input) over its CUDA-event duration, against 148 SMs x 128 lanes x
-          the max SM clock of MEASURED_PEAKS.json.
+roofline: the all-pairs kernel, ALU-pipe bound ("alu"; ncu: the busiest unit):
+          algorithmic ALU-pipe lane-ops per launch (3 per
+          limb-step + 16 per iteration, counted exactly by the kernel's stats
+          pass on the same input) over its CUDA-event duration, against the
+          measured ALU-pipe rate (profiles/r1_pipemix.json) x 32 lanes x SMs x
+          the max SM clock of MEASURED_PEAKS.json; "issue" repeats it for all
+          4 + 16 ops against the measured integer issue ceiling.
 cpu_baseline (rank 0, N = 1): the C oracle (Original Euclid, oracle/) on a
           bounded seeded sample of the same pairs, all host cores.
 --impl reference: the oracle as it stands is the reference arm (no reference
@@ -58,6 +60,7 @@ WORKLOADS = {
 }
 UNIT = "GCD/s"
 OPS_PER_LIMB, OPS_PER_ITER = 4, 16  # SURVEY.md §8(d) M2; DESIGN.md §Roofline
+ALU_OPS_PER_LIMB = 3  # of the 4: IADD3, IADD3.X, SHF.R.W (ALU pipe); IMAD.WIDE.U32 is on the FMA pipe
 
 
 BACKEND = os.environ.get("BULKGCD_BENCH_BACKEND", "nccl")  # "gloo": test mode, ranks may share one GPU
@@ -94,15 +97,50 @@ def _peaks():
         return {"sm_max_mhz": 1965.0}, "fallback"
 
 
-def _int_issue_peak():
-    """Measured integer issue ceiling (tools/intpeak.cu on this pool's B200s,
-    profiles/r1_intpeak.json): ALU + IMAD mix, warp-instructions/clk/SM."""
+def _pipe_rates():
+    """Measured sm_100a issue rates on this pool's B200s (tools/pipemix.cu,
+    profiles/r1_pipemix.json), warp-instructions/clk/SM: the ALU pipe (SHF.R.W
+    alone, the pipe IADD3 carry chains and SHF share) and the best two-pipe mix
+    (the integer issue ceiling)."""
     try:
-        with open(os.path.join(ROOT, "profiles", "r1_intpeak.json")) as f:
-            d = json.load(f)
-        return float(d["ops"]["SHF+IMAD(alu+fma issue probe)"]["warp_inst_per_clk_per_sm_at_max_clock"])
+        with open(os.path.join(ROOT, "profiles", "r1_pipemix.json")) as f:
+            r = json.load(f)["rates"]
+        return float(r["SHF"]), max(float(r["SHF+IMAD"]), float(r["SEL+IMAD"]))
     except (OSError, ValueError, KeyError):
-        return None
+        return None, None
+
+
+def roofline(limbs, iters, n_gcd, kern_s, sms, kernel, share, traffic):
+    """Roofline of the Euclid kernel.  Bound: the ALU pipe (ncu: the
+    busiest unit, profiles/).  Algorithmic ALU-pipe work = 3 lane-ops per limb-step
+    (IADD3 carry-add, IADD3.X borrow, SHF.R.W funnel: the minimal sm_100a limb; its
+    IMAD.WIDE.U32 runs on the FMA pipe in parallel) + 16 per iteration (SURVEY.md
+    §8(d) M2), counted exactly by the kernel's stats pass, over the kernel's
+    CUDA-event time, against the measured ALU-pipe rate x 32 lanes x SMs x the max
+    SM clock (MEASURED_PEAKS.json; NVML shows it held under load).  Also reported:
+    all 4 + 16 ops against the measured integer issue ceiling and the guide's
+    4 warp-instructions/clk/SM."""
+    peaks, src = _peaks()
+    f = float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
+    alu_ipc, issue_ipc = _pipe_rates()
+    src_alu = "measured (profiles/r1_pipemix.json)"
+    if alu_ipc is None:
+        alu_ipc, issue_ipc, src_alu = 2.0, 4.0, "guide unit counts (no pipemix measurement)"
+    alu_ops = (ALU_OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / kern_s
+    all_ops = (OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / kern_s
+    peak = sms * 32 * alu_ipc * f
+    issue_peak = sms * 32 * issue_ipc * f
+    guide = sms * 128 * f
+    return {"bound": "alu", "achieved": alu_ops / 1e12, "peak": peak / 1e12, "unit": "T ALU-pipe lane-ops/s",
+            "frac": alu_ops / peak, "traffic": traffic, "kernel": kernel, "kernel_ms": kern_s * 1e3,
+            "kernel_share_of_step": share,
+            "alu_ops_per_gcd": (ALU_OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / n_gcd,
+            "ops_per_gcd": (OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / n_gcd,
+            "peak_source": (f"ALU pipe {alu_ipc:.3f} warp-instr/clk/SM ({src_alu}) x 32 lanes x {sms} SMs x "
+                            f"{f / 1e6:.0f} MHz ({src} MEASURED_PEAKS sm_max_mhz)"),
+            "issue": {"achieved": all_ops / 1e12, "peak": issue_peak / 1e12, "frac": all_ops / issue_peak,
+                      "unit": "T int lane-ops/s", "ipc": issue_ipc},
+            "peak_guide": guide / 1e12, "frac_of_guide_peak": all_ops / guide}
 
 
 def _traffic():
@@ -292,7 +330,6 @@ def run_pairs(args):
     torch.cuda.synchronize()
     ctr = dS.cpu().numpy().astype(np.int64)
     iters, limbs = int(ctr[2]), int(ctr[4])
-    ops_alg = OPS_PER_LIMB * limbs + OPS_PER_ITER * iters
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
@@ -332,13 +369,8 @@ def run_pairs(args):
         _coll(dist.all_reduce, e2e_t, op=dist.ReduceOp.MAX)
     if rank == 0:
         value = m_all / (step_total_ms / 1e3 / args.steps)
-        peaks, src = _peaks()
-        f_mhz = float(peaks.get("sm_max_mhz", 1965.0))
         sms = torch.cuda.get_device_properties(dev).multi_processor_count
-        ipc = _int_issue_peak() or 4.0
-        peak_ops = sms * 32 * ipc * f_mhz * 1e6
         kern_s = kern_total_ms / 1e3 / args.steps
-        achieved = ops_alg / kern_s
         line = {
             "metric": "1024-bit GCDs/sec (bulk pairs, exact)", "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_total_ms / args.steps,
@@ -349,12 +381,9 @@ def run_pairs(args):
                        "ns_per_gcd": step_total_ms / args.steps * 1e6 / m_all,
                        "iterations_per_gcd": iters / m, "limb_steps_per_gcd": limbs / m,
                        "sample_ok": ok, "sample_checked": int(idx.size)},
-            "roofline": {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
-                         "unit": "T int lane-ops/s", "frac": achieved / peak_ops, "traffic": None,
-                         "kernel": f"pairs_kernel<{W}, exact>", "kernel_ms": kern_s * 1e3,
-                         "kernel_share_of_step": kern_total_ms / step_total_ms, "ops_per_gcd": ops_alg / m,
-                         "hbm_bytes_per_gcd_alg": 3 * W * 4,
-                         "hbm_GBps_alg": 3 * W * 4 * m / kern_s / 1e9},
+            "roofline": dict(roofline(limbs, iters, m, kern_s, sms, f"pairs_kernel<{W}, exact>",
+                                      kern_total_ms / step_total_ms, None),
+                             hbm_bytes_per_gcd_alg=3 * W * 4, hbm_GBps_alg=3 * W * 4 * m / kern_s / 1e9),
             "e2e": {"value": m_all / (float(e2e_t[0]) / args.e2e_steps), "unit": UNIT,
                     "h2d_bytes_per_step": int(A.nbytes + B.nbytes) * world, "d2h_bytes_per_step": int(A.nbytes) * world},
             "gpu_launches": 4 * args.steps,
@@ -473,7 +502,6 @@ def main():
         tt = torch.tensor([iters, limbs], dtype=torch.int64, device=dev)
         _coll(dist.all_reduce, tt)
         iters, limbs = int(tt[0]), int(tt[1])
-    ops_alg = OPS_PER_LIMB * limbs + OPS_PER_ITER * iters  # whole job, per step
 
     k0 = torch.cuda.Event(enable_timing=True)
     k1 = torch.cuda.Event(enable_timing=True)
@@ -545,14 +573,8 @@ def main():
 
     if rank == 0:
         value = pairs / (step_total_ms / 1e3 / args.steps)
-        peaks, src = _peaks()
-        f_mhz = float(peaks.get("sm_max_mhz", 1965.0))
         sms = torch.cuda.get_device_properties(dev).multi_processor_count
-        guide_ops = sms * 128 * f_mhz * 1e6  # lane-ops/s: 4 SMSP x 32 lanes x 1 warp-instr/clk (guide)
-        ipc = _int_issue_peak()
-        peak_ops = sms * 32 * ipc * f_mhz * 1e6 if ipc else guide_ops
         kern_s = kern_total_ms / 1e3 / args.steps
-        achieved = ops_alg / world / kern_s  # per-GPU kernel throughput (each rank runs 1/world of the ops)
         paper = PAPER_GCD_PER_S.get((args.workload, bits))
         line = {
             "metric": metric, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -569,17 +591,10 @@ def main():
                        "ns_per_gcd": step_total_ms / args.steps * 1e6 / pairs,
                        "iterations_per_gcd": iters / pairs, "limb_steps_per_gcd": limbs / pairs,
                        "hits_ok": bool(ok), "hits": len(found), "wall_s": t_wall},
-            "roofline": {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
-                         "unit": "T int lane-ops/s", "frac": achieved / peak_ops, "traffic": _traffic(),
-                         "kernel": f"allpairs_kernel<{W}>" if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
-                         "kernel_ms": kern_s * 1e3,
-                         "kernel_share_of_step": kern_total_ms / step_total_ms,
-                         "ops_per_gcd": ops_alg / pairs,
-                         "peak_source": (f"measured integer issue ceiling {ipc:.3f} warp-instr/clk/SM "
-                                         f"(profiles/r1_intpeak.json) x 32 lanes x {sms} SMs x {f_mhz:.0f} MHz "
-                                         f"({src} MEASURED_PEAKS sm_max_mhz)") if ipc else
-                                        f"{sms} SMs x 128 lanes x {f_mhz:.0f} MHz (guide unit counts)",
-                         "peak_guide": guide_ops / 1e12, "frac_of_guide_peak": achieved / guide_ops},
+            # per-GPU kernel throughput: each rank runs 1/world of the work
+            "roofline": roofline(limbs / world, iters / world, pairs / world, kern_s, sms,
+                                 f"allpairs_kernel<{W}>" if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
+                                 kern_total_ms / step_total_ms, _traffic()),
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,
                     "d2h_bytes_per_step": int(d2h) * world} if e2e_value else None,
             "gpu_launches": 2 * args.steps,

@@ -32,7 +32,36 @@ KEYS = {
     "launch__block_size": "block_size",
     "sm__cycles_elapsed.avg.per_second": "sm_clock_hz",
     "dram__throughput.avg.pct_of_peak_sustained_elapsed": "dram_throughput_pct",
+    "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active": "alu_pipe_cycles_pct",
+    "sm__pipe_fmaheavy_cycles_active.avg.pct_of_peak_sustained_elapsed": "fmaheavy_pipe_cycles_pct",
+    "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active": "fma_pipe_cycles_pct",
 }
+
+
+def opcode_mix(rep):
+    """Executed warp-instructions per SASS opcode (source page), share of the total."""
+    import re
+    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                         capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    hdr = next((r for r in rows if "Source" in r and "Instructions Executed" in r), None)
+    if hdr is None:
+        return {}
+    i_src, i_ex = hdr.index("Source"), hdr.index("Instructions Executed")
+    i_smp = hdr.index("Warp Stall Sampling (All Samples)")
+    cnt, smp = {}, {}
+    for r in rows[rows.index(hdr) + 1:]:
+        m = re.match(r"\s*(@!?U?P\w+\s+)?([A-Z0-9_]+(\.[A-Z0-9_.]+)?)", r[i_src])
+        if not m or not r[i_ex]:
+            continue
+        op = m.group(2)
+        cnt[op] = cnt.get(op, 0) + int(r[i_ex])
+        smp[op] = smp.get(op, 0) + int(r[i_smp] or 0)
+    tot, tots = sum(cnt.values()) or 1, sum(smp.values()) or 1
+    top = sorted(cnt.items(), key=lambda kv: -kv[1])[:24]
+    return {"total_warp_inst": tot, "per_opcode": {k: {"inst_share": round(v / tot, 4),
+                                                       "stall_sample_share": round(smp[k] / tots, 4)}
+                                                   for k, v in top}}
 
 
 def raw(rep):
@@ -84,6 +113,7 @@ def main():
             k = x["Kernel Name"].split("(")[0]
             share[k] = share.get(k, 0.0) + float(x["Metric Value"])
         s["launch_list_share"] = {k: round(v / tot_ns, 5) for k, v in share.items()}
+    s["opcode_mix"] = opcode_mix(rep)
     with open(out, "w") as f:
         json.dump(s, f, indent=1)
     print(json.dumps(s, indent=1))
