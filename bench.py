@@ -584,7 +584,7 @@ def main():
             "config": {"workload": WORKLOADS[args.workload],
                        "n": n, "bits": bits, "pairs": pairs, "mode": "rsa-early-terminate",
                        "algorithm": {"E": "approximate-euclid (register-resident)",
-                                     "D": "fast-binary-euclid (ablation, " + ("register" if bits == 1024 else "smem") + ")",
+                                     "D": "fast-binary-euclid (ablation, smem)",
                                      "C": "binary-euclid (ablation, smem)"}[args.algo],
                        "parallelism": f"row-band x{world}" + (" + NCCL hit all-gather" if world > 1 else ""),
                        "l2": "flushed before every step (256 MiB write); inputs 2 MiB",

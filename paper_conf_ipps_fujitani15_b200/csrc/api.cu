@@ -135,7 +135,7 @@ int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m,
     } else {
     if (flags & (BULKGCD_FLAG_SMEM | BULKGCD_FLAG_ALGO_MASK)) return launch_pairs_smem<W>(a, mode, stats_, flags, st);
     uint64_t cohorts = (m + 31) / 32;
-    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (cohorts + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W, true>::blocks, (cohorts + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
     if (grid == 0) return 0;
     bool stats = (flags & BULKGCD_FLAG_STATS) || d_iters;
     if (mode == BULKGCD_MODE_RSA) {
@@ -185,10 +185,10 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if constexpr (W >= 128) {
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     } else {
-    // (D) on the register harness at 1024 bits (the paper's headline width); other algorithm routes: smem
-    constexpr bool reg_fastbin = W == 32;
-    unsigned algo = flags & BULKGCD_FLAG_ALGO_MASK;
-    if ((flags & BULKGCD_FLAG_SMEM) || (algo && !(reg_fastbin && algo == BULKGCD_FLAG_ALGO_FAST_BINARY)))
+    // the comparison algorithms run on the shared-memory kernels (per-lane pointer swap,
+    // the paper's own design): (D) there measures 661 ms on cfg3 against 1,235 ms on
+    // the register harness, where its frequent no-swap iterations leave the hot loop
+    if ((flags & BULKGCD_FLAG_SMEM) || (flags & BULKGCD_FLAG_ALGO_MASK))
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     uint64_t warps = c1 - c0;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
@@ -197,19 +197,7 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if (!attr_done[0]) {
         CK(cudaFuncSetAttribute(allpairs_kernel<W, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         CK(cudaFuncSetAttribute(allpairs_kernel<W, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        if constexpr (reg_fastbin) {
-            CK(cudaFuncSetAttribute(allpairs_kernel<W, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaFuncSetAttribute(allpairs_kernel<W, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        }
         attr_done[0] = true;
-    }
-    if constexpr (reg_fastbin) {
-        if (algo == BULKGCD_FLAG_ALGO_FAST_BINARY) {
-            if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
-            else allpairs_kernel<W, false, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
-            CK(cudaGetLastError());
-            return 0;
-        }
     }
     if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
     else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, smem, st>>>(a);

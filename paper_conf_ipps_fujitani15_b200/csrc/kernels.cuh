@@ -15,10 +15,16 @@ namespace bulkgcd {
 constexpr int THREADS = BULKGCD_THREADS;
 constexpr int WARPS_PER_CTA = THREADS / 32;
 #ifndef MIN_WARPS
-// resident warps per SM for W <= 32: 16 -> <= 128 registers per thread.  The hot
-// loop stays spill-free (ptxas spills only cold-section state); 16 warps hide the
-// fixed-latency dependency chains better than 12 (cfg3 292 -> 266 ms).
-#define MIN_WARPS 16
+// resident warps per SM for W <= 32: 20 -> <= 96 registers per thread.  ptxas
+// spills cold-section state only; more warps keep the ALU pipe busier across the
+// fixed-latency dependency chains (cfg3: 12 -> 16 warps 292 -> 266 ms, 16 -> 20
+// 253 -> 251 ms).
+#define MIN_WARPS 20
+#endif
+#ifndef MIN_WARPS_PAIRS
+// the exact-mode pairs kernel carries more state (Case-1 tail, L41 normalisation):
+// at 96 registers its spills cost 6.4 -> 11.2 ms on cfg2, so it keeps 16 warps
+#define MIN_WARPS_PAIRS 16
 #endif
 #ifndef MIN_WARPS_W64
 #define MIN_WARPS_W64 8
@@ -28,13 +34,13 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 // Register cap: __launch_bounds__(THREADS, blocks) by default; -DBULKGCD_MAXNREG=N
 // instead caps every kernel at N registers per thread (__maxnreg__).
 #ifdef BULKGCD_MAXNREG
-#define BULKGCD_BOUNDS(W) __maxnreg__(BULKGCD_MAXNREG)
+#define BULKGCD_BOUNDS(W, PAIRS) __maxnreg__(BULKGCD_MAXNREG)
 #else
-#define BULKGCD_BOUNDS(W) __launch_bounds__(THREADS, Occ<W>::blocks)
+#define BULKGCD_BOUNDS(W, PAIRS) __launch_bounds__(THREADS, (Occ<W, PAIRS>::blocks))
 #endif
-template <int W>
+template <int W, bool PAIRS = false>
 struct Occ {
-    static constexpr int warps = W >= 64 ? MIN_WARPS_W64 : MIN_WARPS;
+    static constexpr int warps = W >= 64 ? MIN_WARPS_W64 : (PAIRS ? MIN_WARPS_PAIRS : MIN_WARPS);
     static constexpr int blocks = warps / WARPS_PER_CTA > 0 ? warps / WARPS_PER_CTA : 1;
 };
 
@@ -142,7 +148,7 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
 // and returns true if a finished lane needs cold(...) (warp-converged, with
 // the operand registers); scalar-only finishes are handled by quick itself.
-template <int W, bool STATS, bool EXACT, class Cond, class Sink, class Parker, bool FASTBIN = false>
+template <int W, bool STATS, bool EXACT, class Cond, class Sink, class Parker>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, Parker &pk, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
@@ -194,18 +200,19 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
             }
         }
         bool full, post, lt;
-        hot_iter<W, EXACT, FASTBIN>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
+        hot_iter<W, EXACT>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
         bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
         bool fin = live & !run & !bad;
         bool need = sink.quick_hot(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
-        unsigned bneed = __ballot_sync(FULL, need), btop = __ballot_sync(FULL, top);
-        if (bneed != 0u) {
+        // vote.any with a predicate result: no mask compare on the ALU pipe
+        bool any_need = __any_sync(FULL, need), any_top = __any_sync(FULL, top);
+        if (any_need) {
             fix = fix_code(live, full, post, lt);
             return true;
         }
-        if (btop == 0u) {  // the warp length dropped (lanes finished or shrank): realign one word in place
+        if (!any_top) {  // the warp length dropped (lanes finished or shrank): realign one word in place
             unsigned brun = __ballot_sync(FULL, run);
             // go cold if nobody runs, or to park the last few stragglers (checked only here:
             // the warp length drops when the longest lanes finish)
@@ -429,7 +436,7 @@ struct PairsSinkRsa {
 };
 
 template <int W, bool RSA, bool STATS>
-__global__ void BULKGCD_BOUNDS(W) pairs_kernel(PairsArgs a) {
+__global__ void BULKGCD_BOUNDS(W, true) pairs_kernel(PairsArgs a) {
     const int lane = threadIdx.x & 31;
     uint32_t iters = 0, nslow = 0, limbs = 0, slots = 0, passw = 0;
     for (;;) {
@@ -633,9 +640,8 @@ __device__ __forceinline__ void cohort_coords(uint64_t c, uint64_t n, uint64_t &
     j = 32 * b + 1 + (c - cohorts_before(b, n));
 }
 
-// FASTBIN: the Fast Binary Euclid ablation (N2) on the same register-resident harness.
-template <int W, bool STATS, bool FASTBIN = false>
-__global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
+template <int W, bool STATS>
+__global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     StageBuf<W> *buf = reinterpret_cast<StageBuf<W> *>(smem_raw) + 2 * warp;
@@ -692,7 +698,7 @@ __global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         unsigned K = pk.K;
         if (!allow_park) pk.K = 0;
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, pi, pj};
-        euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk), FASTBIN>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
+        euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
                                      slots, passw);
         pk.K = K;
     };
@@ -730,11 +736,11 @@ __global__ void BULKGCD_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
         if (ParkCfg<W>::on) {
-            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk), FASTBIN>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
+            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
                                          limbs, slots, passw);
         } else {
             NoPark np;
-            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, NoPark, FASTBIN>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
+            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, NoPark>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
                                          limbs, slots, passw);
         }
         slot ^= 1;

@@ -16,7 +16,7 @@ import paper_conf_ipps_fujitani15_b200 as bg  # noqa: E402
 import synth  # noqa: E402
 
 
-def time_allpairs(ms, bits, reps, stats=False):
+def time_allpairs(ms, bits, reps, stats=False, flags=0):
     dev = torch.device("cuda")
     W = bits // 32
     dN = torch.from_numpy(ms.N.view(np.int32)).to(dev)
@@ -27,7 +27,7 @@ def time_allpairs(ms, bits, reps, stats=False):
     dH = torch.zeros(cap * (2 + W), dtype=torch.int32, device=dev)
     dC = torch.zeros(8, dtype=torch.int64, device=dev)
     # stats run
-    bg.bulkgcd_all_pairs_band(dN, dB, ms.m, bits, 0, total, dH, cap, dC, bg.FLAG_STATS)
+    bg.bulkgcd_all_pairs_band(dN, dB, ms.m, bits, 0, total, dH, cap, dC, bg.FLAG_STATS | flags)
     torch.cuda.synchronize()
     ctr = dC.cpu().numpy()
     pairs = ms.m * (ms.m - 1) // 2
@@ -38,7 +38,7 @@ def time_allpairs(ms, bits, reps, stats=False):
     for _ in range(reps):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        bg.bulkgcd_all_pairs_band(dN, dB, ms.m, bits, 0, total, dH, cap, dC, 0)
+        bg.bulkgcd_all_pairs_band(dN, dB, ms.m, bits, 0, total, dH, cap, dC, flags)
         e1.record()
         torch.cuda.synchronize()
         ts.append(e0.elapsed_time(e1) / 1e3)
@@ -82,12 +82,17 @@ def main():
     ap.add_argument("--cfg", type=int, default=3)
     ap.add_argument("--pairs", type=int, default=1 << 18)
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--flags", default="", help="comma list: smem, fastbin, binary")
     a = ap.parse_args()
     print("lib:", os.environ.get("BULKGCD_SO", bg.SO))
     t0 = time.time()
     ms = synth.config_moduli(a.cfg)
     print(f"  generated cfg{a.cfg} in {time.time() - t0:.1f}s")
-    time_allpairs(ms, ms.bits, a.reps)
+    fl = {"smem": bg.FLAG_SMEM, "fastbin": bg.FLAG_ALGO_FAST_BINARY, "binary": bg.FLAG_ALGO_BINARY}
+    flags = 0
+    for f in filter(None, a.flags.split(",")):
+        flags |= fl[f]
+    time_allpairs(ms, ms.bits, a.reps, flags=flags)
     if a.pairs:
         time_pairs(a.pairs, 1024, a.reps, bg.MODE_EXACT)
         time_pairs(a.pairs, 1024, a.reps, bg.MODE_RSA)
