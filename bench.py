@@ -358,11 +358,17 @@ def run_pairs(args):
     step_total_ms, kern_total_ms = float(tot[0]), float(tot[1])
     # e2e: bulkgcd_pairs with host buffers (H2D of A, B; D2H of G inside the call)
     e2e = []
+    # the public path with PINNED host buffers (inputs and result), as an application would stage them
+    pin = lambda a: torch.from_numpy(a.view(np.int32)).pin_memory().numpy().view(np.uint32)
+    A, B = pin(A), pin(B)
+    Gh = torch.empty(A.shape, dtype=torch.int32).pin_memory().numpy().view(np.uint32)
+    if args.e2e_steps:  # one untimed warm-up call of the public path
+        bg.bulkgcd_pairs(A, B, bits, out=Gh)
     for _ in range(args.e2e_steps):
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
-        bg.bulkgcd_pairs(A, B, bits)
+        bg.bulkgcd_pairs(A, B, bits, out=Gh)
         e2e.append(time.perf_counter() - t0)
     e2e_t = torch.tensor([sum(e2e)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -553,6 +559,8 @@ def main():
     d2h = 0
     if args.algo != "E":
         args.e2e_steps = 0  # the public API runs (E); an ablation has no end-to-end line
+    if args.e2e_steps:  # one untimed warm-up call of the public path (allocator pools, lazy module loading)
+        bg.bulkgcd_all_pairs(Nh, bits) if world == 1 else bgd.all_pairs_distributed(Nh, bits)
     for _ in range(args.e2e_steps):
         flush.fill_(3)
         torch.cuda.synchronize()

@@ -27,7 +27,9 @@
  * Threading.  Reentrant; host entry points use the calling thread's
  * per-thread default CUDA stream and stream-ordered allocations, inputs are
  * never modified, and there is no global state besides a thread-local error
- * message.
+ * message and, once per device, a release threshold of 4 GiB on the device's
+ * default memory pool (stream-ordered buffers stay cached between calls
+ * instead of being unmapped at every synchronisation).
  */
 #ifndef BULKGCD_H
 #define BULKGCD_H

@@ -120,19 +120,26 @@ def _stream(stream) -> int | None:
 
 
 # ------------------------------------------------------------- host entry points
-def bulkgcd_pairs(A, B, bits: int) -> np.ndarray:
-    """G[i] = gcd(A[i], B[i]) (exact mode).  A, B: uint32[m, bits/32]."""
-    G, _ = bulkgcd_pairs_ex(A, B, bits, MODE_EXACT, want_iters=False)
+def bulkgcd_pairs(A, B, bits: int, out: np.ndarray | None = None) -> np.ndarray:
+    """G[i] = gcd(A[i], B[i]) (exact mode).  A, B: uint32[m, bits/32].  `out`: an
+    optional caller-owned result array of the same shape (e.g. pinned host memory)."""
+    G, _ = bulkgcd_pairs_ex(A, B, bits, MODE_EXACT, want_iters=False, out=out)
     return G
 
 
-def bulkgcd_pairs_ex(A, B, bits: int, mode: int = MODE_EXACT, want_iters: bool = False):
+def bulkgcd_pairs_ex(A, B, bits: int, mode: int = MODE_EXACT, want_iters: bool = False,
+                     out: np.ndarray | None = None):
     W = _words(bits)
     A, B = _host(A, W), _host(B, W)
     if A.shape != B.shape:
         raise ValueError("A and B must have the same shape")
     m = A.shape[0]
-    G = np.zeros_like(A)
+    if out is None:
+        G = np.zeros_like(A)
+    else:
+        G = out
+        if G.dtype != np.uint32 or G.shape != A.shape or not G.flags.c_contiguous:
+            raise ValueError(f"out must be a C-contiguous uint32{list(A.shape)} array")
     it = np.zeros(m, np.uint32) if want_iters else None
     _check(lib().bulkgcd_pairs_ex(A.ctypes.data, B.ctypes.data, m, bits, mode, G.ctypes.data,
                                   it.ctypes.data if it is not None else None))

@@ -66,6 +66,19 @@ int device_check() {
     if (major != 10 || minor != 0)
         return set_err(BULKGCD_ENODEV, "device %d is sm_%d%d; libbulkgcd is built for sm_100a only", dev, major,
                        minor);
+    // The host-buffer entry points allocate stream-ordered (cudaMallocAsync) per call; by
+    // default the pool unmaps everything at each synchronisation, so a repeated call
+    // re-maps its buffers (hundreds of MB for bulkgcd_pairs).  Keep up to 4 GiB cached
+    // in the device's default pool (the per-device context of include/bulkgcd.h B5).
+    static bool pool_set[64] = {};  // idempotent, benign race
+    if (dev < 64 && !pool_set[dev]) {
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t keep = 4ull << 30;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+        }
+        pool_set[dev] = true;
+    }
     return 0;
 }
 

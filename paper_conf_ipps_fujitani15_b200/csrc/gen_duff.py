@@ -97,10 +97,95 @@ def emit(W: int, form: str = "split", G: int = 1) -> str:
     return "\n".join(o)
 
 
+def emit_two(W: int, G: int) -> str:
+    """Two-borrow-chain form: Z = X - lo(alpha*Y) - hi(alpha*Y)*D, per G-limb block
+    chain 1 subtracts the low product words, chain 2 the high words one limb up
+    (tools/limbmix.cu: no carry-add / IMAD.X per limb; 9.5 -> 8.9 SMSP-cycles per
+    limb in isolation at G = 8).  The borrows cross block boundaries through two
+    registers (save: subc 0,0 -> 0 or -1; restore: sub.cc 0, b)."""
+    xa = lambda k: "%%%d" % (2 + k)
+    ya = lambda k: "%%%d" % (W + 2 + k)
+    al = "%%%d" % (2 * W + 2)
+    sa = "%%%d" % (2 * W + 3)
+    regs = ", ".join([f"l{g}, h{g}, z{g}" for g in range(G)])
+    a = ["{", f".reg .u32 zp, hp, b1, b2, t, {regs};", ".reg .u64 p;", ".reg .pred pe;",
+         "setp.ge.s32 pe, %s, 0;" % sa,
+         "ts: .branchtargets %s;" % ", ".join("E%d" % k for k in range(W)),
+         "brx.idx %s, ts;" % sa]
+
+    def block(k0, k1, head):
+        """limbs k0..k1-1 (one G-block or the head's partial block)."""
+        n = k1 - k0
+        out = []
+        for g in range(n):
+            out += ["mul.wide.u32 p, %s, %s;" % (al, ya(k0 + g)), f"mov.b64 {{l{g}, h{g}}}, p;"]
+        # chain 1: z = x - lo
+        if head:
+            out.append("sub.cc.u32 z0, %s, l0;" % xa(k0))
+        else:
+            out += ["sub.cc.u32 t, 0, b1;", "subc.cc.u32 z0, %s, l0;" % xa(k0)]
+        for g in range(1, n):
+            out.append(f"subc.cc.u32 z{g}, %s, l{g};" % xa(k0 + g))
+        out.append("subc.u32 b1, 0, 0;")
+        if head:  # r = ctz(z_s): chain 2 does not touch the first limb
+            out += ["mov.u32 %1, z0;", "brev.b32 t, z0;", "clz.b32 %0, t;"]
+        # chain 2: z -= hi one limb up (hp = hi of the limb below the block)
+        if head:
+            if n > 1:
+                out.append("sub.cc.u32 z1, z1, h0;")
+                for g in range(2, n):
+                    out.append(f"subc.cc.u32 z{g}, z{g}, h{g - 1};")
+                out.append("subc.u32 b2, 0, 0;")
+            else:
+                out.append("mov.u32 b2, 0;")
+        else:
+            out += ["sub.cc.u32 t, 0, b2;", "subc.cc.u32 z0, z0, hp;"]
+            for g in range(1, n):
+                out.append(f"subc.cc.u32 z{g}, z{g}, h{g - 1};")
+            out.append("subc.u32 b2, 0, 0;")
+        out.append(f"mov.u32 hp, h{n - 1};")
+        # funnel shifts: X[k-1] = (z_{k-1}, z_k) >> r
+        for g in range(n):
+            k = k0 + g
+            if head and g == 0:
+                pass
+            else:
+                out.append(f"shf.r.wrap.b32 %s, zp, z{g}, %%0;" % xa(k - 1))
+            out.append(f"mov.u32 zp, z{g};")
+        return out
+
+    for k in range(W):
+        e = min((k // G + 1) * G, W)
+        nxt = "B%d" % e if e < W else "TOP"
+        a.append("E%d:" % k)
+        a += block(k, e, True)
+        a.append("@pe bra %s;" % nxt)
+    a.append("bra.uni TOP;")
+    for k in range(G, W, G):
+        a.append("B%d:" % k)
+        a += block(k, min(k + G, W), False)
+    a += ["TOP:", "shf.r.wrap.b32 %s, zp, 0, %%0;" % xa(W - 1), "}"]
+    body = "\\n\\t".join(x.replace('"', '\\"') for x in a)
+    outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(X[%d])' % k for k in range(W)]
+    ins = ['"r"(Y[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)']
+    o = ["template <>",
+         "__device__ __forceinline__ uint32_t duff_pass<%d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
+         "uint32_t alpha, int s, uint32_t &r) {" % (W, W, W),
+         "  uint32_t zs;",
+         '  asm volatile("%s"' % body,
+         "      : %s" % ", ".join(outs),
+         "      : %s);" % ", ".join(ins),
+         "  return zs;",
+         "}"]
+    return "\n".join(o)
+
+
 def main():
     import sys
     form = sys.argv[1] if len(sys.argv) > 1 else os.environ.get("BULKGCD_PASS_FORM", "split")
     G = int(os.environ.get("BULKGCD_PASS_G", "4"))
+    if form == "two":
+        G = int(os.environ.get("BULKGCD_PASS_G", "8"))
     here = os.path.dirname(os.path.abspath(__file__))
     parts = [
         "// GENERATED by gen_duff.py -- do not edit by hand.",
@@ -120,10 +205,11 @@ def main():
         "",
     ]
     for W in WIDTHS:
-        parts.append(emit(W, form, G))
+        parts.append(emit_two(W, G) if form == "two" else emit(W, form, G))
         parts.append("")
     parts.append("}  // namespace bulkgcd")
-    with open(os.path.join(here, "duff_pass.cuh"), "w") as f:
+    out = os.environ.get("BULKGCD_DUFF_OUT", os.path.join(here, "duff_pass.cuh"))
+    with open(out, "w") as f:
         f.write("\n".join(parts) + "\n")
 
 

@@ -57,6 +57,12 @@ def test_host_validation_no_gpu_needed(bg):
     assert e.value.code == bg.EINVAL
     # m = 0 / n < 2 are no-ops
     assert bg.bulkgcd_pairs(np.zeros((0, W), np.uint32), np.zeros((0, W), np.uint32), 1024).shape == (0, W)
+    # a caller-owned result buffer must match the operands
+    for bad in (np.zeros((3, W), np.uint32), np.zeros((2, W), np.int64), np.zeros((W, 2), np.uint32).T):
+        with pytest.raises(ValueError):
+            bg.bulkgcd_pairs(Z, Z, 1024, out=bad)
+    out = np.zeros((0, W), np.uint32)
+    assert bg.bulkgcd_pairs(Z[:0], Z[:0], 1024, out=out) is out
     one = np.zeros((1, W), np.uint32)
     one[0, 0] = 3
     assert bg.bulkgcd_all_pairs(one, 1024).ij.shape == (0, 2)

@@ -22,10 +22,15 @@ def main():
         so = os.path.join(OUT, f"libbulkgcd_{name}.so")
         toks = shlex.split(flags)
         env = dict(t[4:].split("=", 1) for t in toks if t.startswith("env:"))  # env:KEY=VAL -> gen_duff settings
+        extra = [t for t in toks if not t.startswith("env:")]
+        if env:  # the variant's own generated pass (parallel variant builds do not race on csrc/duff_pass.cuh)
+            hdr = os.path.join(OUT, f"duff_pass_{name}.cuh")
+            env["BULKGCD_DUFF_OUT"] = hdr
+            extra.append(f'-DBULKGCD_DUFF_HEADER="{hdr}"')
         saved = {k: os.environ.get(k) for k in env}
         os.environ.update(env)
         try:
-            _build.build(out=so, extra_flags=[t for t in toks if not t.startswith("env:")])
+            _build.build(out=so, extra_flags=extra)
         finally:
             for k, v in saved.items():
                 if v is None:
