@@ -316,6 +316,60 @@ int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t 
     }
 }
 
+// Large host-buffer batches run in chunks on two streams, so the copy engines move chunk
+// c+1 in (and chunk c-1 out) while chunk c computes: H2D, layout, kernel, layout back
+// and D2H of one chunk are ordered on its stream, and a stream's buffers are reused by
+// its next chunk only after its D2H (stream order).  Overlap needs pinned host buffers;
+// with pageable ones the driver stages the copies synchronously and the result is the same.
+constexpr size_t PAIRS_CHUNK = size_t(1) << 18;
+
+struct StreamPair {
+    cudaStream_t s[2] = {nullptr, nullptr};
+    ~StreamPair() {
+        for (auto &x : s)
+            if (x) cudaStreamDestroy(x);
+    }
+};
+
+static int pairs_chunked(const uint32_t *A, const uint32_t *B, size_t m, int W, uint32_t bits, int mode, uint32_t *G,
+                         uint32_t *iters) {
+    StreamPair sp;
+    for (auto &x : sp.s) CK(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+    const size_t rm = PAIRS_CHUNK * W * 4, cm = pad32(PAIRS_CHUNK) * W * 4;
+    struct Bufs {
+        DBuf a, b, ac, bc, gc, it, sc;
+    } buf[2];
+    for (int k = 0; k < 2; ++k) {
+        cudaStream_t st = sp.s[k];
+        CK(buf[k].a.alloc(rm, st));
+        CK(buf[k].b.alloc(rm, st));
+        CK(buf[k].ac.alloc(cm, st));
+        CK(buf[k].bc.alloc(cm, st));
+        CK(buf[k].gc.alloc(cm, st));
+        CK(buf[k].sc.alloc(8 * sizeof(unsigned long long), st));
+        if (iters) CK(buf[k].it.alloc(PAIRS_CHUNK * 4, st));
+    }
+    int rc;
+    for (size_t c = 0, off = 0; off < m; ++c, off += PAIRS_CHUNK) {
+        Bufs &b = buf[c & 1];
+        cudaStream_t st = sp.s[c & 1];
+        size_t mc = std::min(PAIRS_CHUNK, m - off), mp = pad32(mc), bytes = mc * W * 4;
+        CK(cudaMemcpyAsync(b.a.p, A + off * W, bytes, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(b.b.p, B + off * W, bytes, cudaMemcpyHostToDevice, st));
+        if ((rc = bulkgcd_interleave(b.a.as<uint32_t>(), b.ac.as<uint32_t>(), mc, mp, bits, 1, st))) return rc;
+        if ((rc = bulkgcd_interleave(b.b.as<uint32_t>(), b.bc.as<uint32_t>(), mc, mp, bits, 1, st))) return rc;
+        if ((rc = bulkgcd_pairs_device(b.ac.as<uint32_t>(), b.bc.as<uint32_t>(), b.gc.as<uint32_t>(), mc, mp, bits,
+                                       mode, iters ? b.it.as<uint32_t>() : nullptr, b.sc.as<unsigned long long>(),
+                                       0, st)))
+            return rc;
+        if ((rc = bulkgcd_interleave(b.gc.as<uint32_t>(), b.a.as<uint32_t>(), mc, mp, bits, 0, st))) return rc;
+        CK(cudaMemcpyAsync(G + off * W, b.a.p, bytes, cudaMemcpyDeviceToHost, st));
+        if (iters) CK(cudaMemcpyAsync(iters + off, b.it.p, mc * 4, cudaMemcpyDeviceToHost, st));
+    }
+    for (auto &x : sp.s) CK(cudaStreamSynchronize(x));
+    return 0;
+}
+
 int bulkgcd_pairs_ex(const uint32_t *A, const uint32_t *B, size_t m, uint32_t bits, int mode, uint32_t *G,
                      uint32_t *iters) {
     int W = words_for(bits);
@@ -330,6 +384,7 @@ int bulkgcd_pairs_ex(const uint32_t *A, const uint32_t *B, size_t m, uint32_t bi
     }
     int rc = device_check();
     if (rc) return rc;
+    if (m > PAIRS_CHUNK) return pairs_chunked(A, B, m, W, bits, mode, G, iters);
     cudaStream_t st = cudaStreamPerThread;
     size_t m_pad = pad32(m), rm = m * W * 4, cm = m_pad * W * 4;
     DBuf dA, dB, dAc, dBc, dGc, dIt, dS;

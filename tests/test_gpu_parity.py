@@ -224,6 +224,58 @@ def test_all_pairs_config3_full(bg):
         assert oracle.gcd(synth.to_int(ms.N[a]), synth.to_int(ms.N[b])) == g
 
 
+def test_all_pairs_config4_full(bg):
+    """BASELINE configs[3] (2048-bit, 16,384 moduli) at full size: exact hit set
+    against construction ground truth, plus a seeded sample through the oracle."""
+    ms = synth.config_moduli(4)
+    assert ms.bits == 2048
+    hits = bg.bulkgcd_all_pairs(ms.N, 2048).as_list()
+    assert hits == ms.truth
+    rng = np.random.default_rng(4)
+    ii = rng.integers(0, ms.m, size=6000)
+    jj = rng.integers(0, ms.m, size=6000)
+    keep = ii < jj
+    ii, jj = ii[keep], jj[keep]
+    hit = oracle.rsa_hit(oracle.bitlen_rows(oracle.gcd_index_pairs(ms.N, ii, jj)), 2048)
+    truth = {(a, b) for a, b, _ in ms.truth}
+    assert [bool(h) for h in hit] == [(int(a), int(b)) in truth for a, b in zip(ii, jj)]
+
+
+def test_all_pairs_config5_full(bg):
+    """BASELINE configs[4] (65,536 moduli, 2,147,450,880 pairs) on one GPU: the
+    exact hit set (33 planted pairs) against construction ground truth."""
+    ms = synth.config_moduli(5)
+    hits = bg.bulkgcd_all_pairs(ms.N, 1024).as_list()
+    assert len(ms.truth) == 33 and hits == ms.truth
+
+
+def test_pairs_config2_full_bit_exact(bg):
+    """BASELINE configs[1] at full size (2^20 exact-mode pairs, the bench's launch):
+    every gcd bit-exact against the oracle's classical Euclid."""
+    A, B, _ = synth.config2()
+    G = bg.bulkgcd_pairs(A, B, 1024)
+    want = oracle.gcd_batch(A, B)
+    assert G.shape == want.shape and np.array_equal(G, want)
+    assert int((oracle.bitlen_rows(G) > 1).sum()) >= 2  # the planted pairs are among them
+
+
+def test_pairs_chunked_host_path(bg):
+    """Host batches above 2^18 pairs run in overlapped chunks on two streams:
+    gcds and per-pair iteration counts equal single-chunk calls on the same
+    pairs (ragged last chunk, both modes), and the gcds equal the oracle on a
+    sample."""
+    A, B, _ = synth.config2(3 * (1 << 18) + 777)
+    for mode in (bg.MODE_EXACT, bg.MODE_RSA):
+        G, it = bg.bulkgcd_pairs_ex(A, B, 1024, mode, want_iters=True)
+        for lo in (0, 1 << 18, 3 * (1 << 18)):
+            hi = min(lo + 100_000, A.shape[0])
+            g1, it1 = bg.bulkgcd_pairs_ex(A[lo:hi], B[lo:hi], 1024, mode, want_iters=True)
+            assert np.array_equal(G[lo:hi], g1) and np.array_equal(it[lo:hi], it1)
+    idx = np.random.default_rng(5).integers(0, A.shape[0], 4000)
+    G = bg.bulkgcd_pairs(A, B, 1024)
+    assert np.array_equal(G[idx], oracle.gcd_batch(A[idx], B[idx]))
+
+
 def _dist_worker(rank, world, port, out):
     import os
     import torch.distributed as dist
