@@ -27,7 +27,13 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 #define MIN_WARPS_PAIRS 16
 #endif
 #ifndef MIN_WARPS_W64
-#define MIN_WARPS_W64 8
+// W = 64 all-pairs: 12 warps/SM (168 registers; ptxas spills ~4 KB of cold and window state)
+// beat 8 warps (255 registers, spill-free): cfg4 1,034 -> 943 ms; 16 warps spill the
+// operands themselves (1,708 ms).  The pairs kernel keeps 8 (not measured at 12).
+#define MIN_WARPS_W64 12
+#endif
+#ifndef MIN_WARPS_W64_PAIRS
+#define MIN_WARPS_W64_PAIRS 8
 #endif
 // CTAs per SM by width: the operands take 2W registers per thread; W = 64
 // (2048-bit) needs ~200+ registers, i.e. 8 warps per SM.
@@ -40,7 +46,8 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 #endif
 template <int W, bool PAIRS = false>
 struct Occ {
-    static constexpr int warps = W >= 64 ? MIN_WARPS_W64 : (PAIRS ? MIN_WARPS_PAIRS : MIN_WARPS);
+    static constexpr int warps = W >= 64 ? (PAIRS ? MIN_WARPS_W64_PAIRS : MIN_WARPS_W64)
+                                         : (PAIRS ? MIN_WARPS_PAIRS : MIN_WARPS);
     static constexpr int blocks = warps / WARPS_PER_CTA > 0 ? warps / WARPS_PER_CTA : 1;
 };
 
