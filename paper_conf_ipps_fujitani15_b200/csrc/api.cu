@@ -194,7 +194,7 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
                     uint64_t cap, unsigned long long *counters, unsigned flags, cudaStream_t st) {
     CK(cudaMemsetAsync(counters, 0, 8 * sizeof(unsigned long long), st));
     if (c1 <= c0) return 0;
-    AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
+    AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16, nullptr};
     if constexpr (W >= 128) {
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     } else {
@@ -205,6 +205,11 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     uint64_t warps = c1 - c0;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
+    DBuf park;  // freed stream-ordered after the kernel
+    if constexpr (ParkCfg<W>::gmem) {
+        CK(park.alloc(grid * WARPS_PER_CTA * sizeof(ParkPool<W>), st));
+        a.park = park.p;
+    }
     constexpr size_t smem = allpairs_smem_bytes<W>();
     static bool attr_done[2] = {false, false};  // idempotent, benign race
     if (!attr_done[0]) {

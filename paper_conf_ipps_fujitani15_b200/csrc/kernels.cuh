@@ -544,6 +544,7 @@ struct AllPairsArgs {
     unsigned long long *hit_count;
     unsigned long long *stats;     // optional [sum iterations, slow steps, limb-steps]
     int half;
+    void *park;                    // straggler pools in global memory (ParkCfg<W>::gmem), one per warp
 };
 
 template <int W>
@@ -594,11 +595,16 @@ struct StageBuf {
 #ifndef BULKGCD_PARK_K
 #define BULKGCD_PARK_K 0  // straggler parking: measured a wash on B200, off by default
 #endif
-// Parking pool only where it fits next to the TMA buffers at the kernel's occupancy.
+#ifndef BULKGCD_PARK_GMEM
+#define BULKGCD_PARK_GMEM 1  // pool in global memory (per warp, L2-resident), not next to the TMA buffers
+#endif
+// Parking pool: in shared memory only where it fits next to the TMA buffers at the
+// kernel's occupancy; in global memory (AllPairsArgs::park, one pool per warp) otherwise.
 template <int W>
 struct ParkCfg {
-    static constexpr bool on = (W <= 32) && (BULKGCD_PARK_K > 0);
-    static constexpr size_t pool_bytes = on ? sizeof(ParkPool<W>) : 0;
+    static constexpr bool on = (BULKGCD_PARK_GMEM ? W <= 64 : W <= 32) && (BULKGCD_PARK_K > 0);
+    static constexpr bool gmem = on && BULKGCD_PARK_GMEM;
+    static constexpr size_t pool_bytes = (on && !gmem) ? sizeof(ParkPool<W>) : 0;
 };
 
 template <int W>
@@ -653,7 +659,9 @@ __global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     StageBuf<W> *buf = reinterpret_cast<StageBuf<W> *>(smem_raw) + 2 * warp;
     unsigned char *after_bufs = smem_raw + (THREADS / 32) * 2 * sizeof(StageBuf<W>);
-    ParkPool<W> *pool = reinterpret_cast<ParkPool<W> *>(after_bufs) + warp;  // valid only if ParkCfg<W>::on
+    ParkPool<W> *pool = ParkCfg<W>::gmem  // valid only if ParkCfg<W>::on
+                            ? reinterpret_cast<ParkPool<W> *>(a.park) + (blockIdx.x * (THREADS / 32) + warp)
+                            : reinterpret_cast<ParkPool<W> *>(after_bufs) + warp;
     unsigned long long *bar =
         reinterpret_cast<unsigned long long *>(after_bufs + (THREADS / 32) * ParkCfg<W>::pool_bytes) + 2 * warp;
     if (lane == 0) {
