@@ -45,7 +45,7 @@ sys.path.insert(0, ROOT)
 
 # The paper's GTX 780 Ti, early-terminate, all pairs of 16K moduli (Table V):
 # 0.346 us/GCD at 1024 bits, 1.33 us/GCD at 2048 bits.  Same workload size as cfg3 / cfg4.
-PAPER_GCD_PER_S = {("cfg3", 1024): 1.0 / 0.346e-6, ("cfg4", 2048): 1.0 / 1.33e-6}
+PAPER_GCD_PER_S = {("cfg3", 1024): 1.0 / 0.346e-6, ("cfg4", 2048): 1.0 / 1.33e-6, ("cfg6", 512): 1.0 / 0.0773e-6}
 METRIC = "1024-bit GCDs/sec (all-pairs)"
 WORKLOADS = {
     "cfg1": "cfg1: all-pairs 1024-bit RSA moduli, n=64 (2,016 pairs), 3 planted shared primes (BASELINE.json configs[0])",
@@ -55,6 +55,10 @@ WORKLOADS = {
             "(BASELINE.json configs[3])",
     "cfg5": "cfg5: all-pairs 1024-bit RSA moduli, n=65536 (2,147,450,880 pairs), 33 planted shared primes "
             "(BASELINE.json configs[4])",
+    "cfg6": "cfg6: all-pairs 512-bit RSA moduli, n=16384 (134,209,536 pairs), 8 planted shared primes "
+            "(the paper's 512-bit Table V workload; SURVEY.md §8(f) N1, not a BASELINE.json config)",
+    "cfg7": "cfg7: all-pairs 4096-bit RSA moduli, n=512 (130,816 pairs), 4 planted shared primes "
+            "(shared-memory kernels; SURVEY.md §8(f) N1, not a BASELINE.json config)",
     "cfg2": "cfg2: 2^20 independent 1024-bit pair GCDs, exact mode (bulkgcd_pairs; the first 2^20 pairs i<j "
             "of a 1,449-moduli pool with 2 planted shared primes; BASELINE.json configs[1])",
 }
@@ -591,7 +595,7 @@ def main():
             "data": "synthetic",
             "config": {"workload": WORKLOADS[args.workload],
                        "n": n, "bits": bits, "pairs": pairs, "mode": "rsa-early-terminate",
-                       "algorithm": {"E": "approximate-euclid (register-resident)",
+                       "algorithm": {"E": "approximate-euclid (" + ("register" if W < 128 else "shared-memory") + "-resident)",
                                      "D": "fast-binary-euclid (ablation, smem)",
                                      "C": "binary-euclid (ablation, smem)"}[args.algo],
                        "parallelism": f"row-band x{world}" + (" + NCCL hit all-gather" if world > 1 else ""),
@@ -601,7 +605,8 @@ def main():
                        "hits_ok": bool(ok), "hits": len(found), "wall_s": t_wall},
             # per-GPU kernel throughput: each rank runs 1/world of the work
             "roofline": roofline(limbs / world, iters / world, pairs / world, kern_s, sms,
-                                 f"allpairs_kernel<{W}>" if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
+                                 (f"allpairs_kernel<{W}>" if W < 128 else f"allpairs_smem_kernel<{W}>")
+                                 if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
                                  kern_total_ms / step_total_ms, _traffic()),
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,
                     "d2h_bytes_per_step": int(d2h) * world} if e2e_value else None,

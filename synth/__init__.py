@@ -188,6 +188,9 @@ CONFIGS = {
     3: dict(m=16384, bits=1024, n_planted_pairs=8),
     4: dict(m=16384, bits=2048, n_planted_pairs=8),
     5: dict(m=65536, bits=1024, n_planted_pairs=33),
+    # the paper's other Table V widths (not BASELINE.json configs)
+    6: dict(m=16384, bits=512, n_planted_pairs=8),
+    7: dict(m=512, bits=4096, n_planted_pairs=4),
 }
 CFG2_POOL = 1449          # 1449*1448/2 = 1,049,076 >= 2^20 pairs
 CFG2_PAIRS = 1 << 20
