@@ -21,6 +21,9 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 // 253 -> 251 ms).
 #define MIN_WARPS 20
 #endif
+#ifndef MIN_WARPS_W16
+#define MIN_WARPS_W16 32  // 512-bit all-pairs: 64 registers (cfg6 86.4 -> 84.8 ms against 20 warps)
+#endif
 #ifndef MIN_WARPS_PAIRS
 // the exact-mode pairs kernel carries more state (Case-1 tail, L41 normalisation):
 // at 96 registers its spills cost 6.4 -> 11.2 ms on cfg2, so it keeps 16 warps
@@ -29,11 +32,11 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 #ifndef MIN_WARPS_W64
 // W = 64 all-pairs: 12 warps/SM (168 registers; ptxas spills ~4 KB of cold and window state)
 // beat 8 warps (255 registers, spill-free): cfg4 1,034 -> 943 ms; 16 warps spill the
-// operands themselves (1,708 ms).  The pairs kernel keeps 8 (not measured at 12).
+// operands themselves (1,708 ms).
 #define MIN_WARPS_W64 12
 #endif
 #ifndef MIN_WARPS_W64_PAIRS
-#define MIN_WARPS_W64_PAIRS 8
+#define MIN_WARPS_W64_PAIRS 12  // 2048-bit pairs: 2^18 exact 7.67 -> 7.23 ms, RSA 3.58 -> 3.29 ms against 8
 #endif
 // CTAs per SM by width: the operands take 2W registers per thread; W = 64
 // (2048-bit) needs ~200+ registers, i.e. 8 warps per SM.
@@ -47,7 +50,7 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 template <int W, bool PAIRS = false>
 struct Occ {
     static constexpr int warps = W >= 64 ? (PAIRS ? MIN_WARPS_W64_PAIRS : MIN_WARPS_W64)
-                                         : (PAIRS ? MIN_WARPS_PAIRS : MIN_WARPS);
+                                         : (PAIRS ? MIN_WARPS_PAIRS : (W <= 16 ? MIN_WARPS_W16 : MIN_WARPS));
     static constexpr int blocks = warps / WARPS_PER_CTA > 0 ? warps / WARPS_PER_CTA : 1;
 };
 

@@ -51,7 +51,13 @@ def time_allpairs(ms, bits, reps, stats=False, flags=0):
 def time_pairs(m, bits, reps, mode):
     dev = torch.device("cuda")
     W = bits // 32
-    A, B, _ = synth.config2(m)
+    if bits == 1024:
+        A, B, _ = synth.config2(m)
+    else:  # the first m pairs (i < j) of a seeded pool at this width
+        pool = int((1 + (1 + 8 * m) ** 0.5) / 2) + 1
+        ms = synth.moduli(pool, bits, 4242, n_planted_pairs=2)
+        i, j = synth.pair_indices(pool, m)
+        A, B = ms.N[i], ms.N[j]
     m_pad = (m + 31) // 32 * 32
     dA = torch.from_numpy(A.view(np.int32)).to(dev)
     dB = torch.from_numpy(B.view(np.int32)).to(dev)
@@ -83,6 +89,7 @@ def main():
     ap.add_argument("--pairs", type=int, default=1 << 18)
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--flags", default="", help="comma list: smem, fastbin, binary")
+    ap.add_argument("--pair-bits", type=int, default=1024)
     a = ap.parse_args()
     print("lib:", os.environ.get("BULKGCD_SO", bg.SO))
     t0 = time.time()
@@ -94,8 +101,8 @@ def main():
         flags |= fl[f]
     time_allpairs(ms, ms.bits, a.reps, flags=flags)
     if a.pairs:
-        time_pairs(a.pairs, 1024, a.reps, bg.MODE_EXACT)
-        time_pairs(a.pairs, 1024, a.reps, bg.MODE_RSA)
+        time_pairs(a.pairs, a.pair_bits, a.reps, bg.MODE_EXACT)
+        time_pairs(a.pairs, a.pair_bits, a.reps, bg.MODE_RSA)
 
 
 if __name__ == "__main__":
