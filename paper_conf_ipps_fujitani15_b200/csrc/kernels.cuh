@@ -25,9 +25,9 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 #define MIN_WARPS_W16 32  // 512-bit all-pairs: 64 registers (cfg6 86.4 -> 84.8 ms against 20 warps)
 #endif
 #ifndef MIN_WARPS_PAIRS
-// the exact-mode pairs kernel carries more state (Case-1 tail, L41 normalisation):
-// at 96 registers its spills cost 6.4 -> 11.2 ms on cfg2, so it keeps 16 warps
-#define MIN_WARPS_PAIRS 16
+// the pairs kernel (1024-bit, 2^20 pairs): 16 -> 20 warps exact 4.22 -> 4.19 ms, RSA 3.65 -> 3.32 ms;
+// 24 warps 4.32 / 3.47 ms
+#define MIN_WARPS_PAIRS 20
 #endif
 #ifndef MIN_WARPS_W64
 // W = 64 all-pairs: 12 warps/SM (168 registers; ptxas spills ~4 KB of cold and window state)
