@@ -210,8 +210,8 @@ def test_all_pairs_config3_full(bg):
     hits = bg.bulkgcd_all_pairs(ms.N, 1024).as_list()
     assert hits == ms.truth
     rng = np.random.default_rng(3)
-    ii = rng.integers(0, ms.m, size=20000)
-    jj = rng.integers(0, ms.m, size=20000)
+    ii = rng.integers(0, ms.m, size=400_000)
+    jj = rng.integers(0, ms.m, size=400_000)
     keep = ii < jj
     ii, jj = ii[keep], jj[keep]
     G = oracle.gcd_index_pairs(ms.N, ii, jj)
@@ -232,8 +232,8 @@ def test_all_pairs_config4_full(bg):
     hits = bg.bulkgcd_all_pairs(ms.N, 2048).as_list()
     assert hits == ms.truth
     rng = np.random.default_rng(4)
-    ii = rng.integers(0, ms.m, size=6000)
-    jj = rng.integers(0, ms.m, size=6000)
+    ii = rng.integers(0, ms.m, size=60_000)
+    jj = rng.integers(0, ms.m, size=60_000)
     keep = ii < jj
     ii, jj = ii[keep], jj[keep]
     hit = oracle.rsa_hit(oracle.bitlen_rows(oracle.gcd_index_pairs(ms.N, ii, jj)), 2048)
