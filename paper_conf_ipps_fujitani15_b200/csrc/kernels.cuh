@@ -158,7 +158,7 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
 // and returns true if a finished lane needs cold(...) (warp-converged, with
 // the operand registers); scalar-only finishes are handled by quick itself.
-template <int W, bool STATS, bool EXACT, class Cond, class Sink, class Parker>
+template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, class Parker>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, Parker &pk, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
@@ -241,7 +241,15 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
     for (;;) {
         bool more = resume == 0 ? cold(A, B, lA, tA, lB, tB) : cold(B, A, lB, tB, lA, tA);
         if (!more) return;
-        if (resume == 1) {
+        // ONE_ENTRY: resuming on roles (B, A) enters the loop at its second hot
+        // iteration, so the pass is inlined twice (once per role assignment) instead of
+        // three times.  Measured: RSA pairs 3.30 -> 2.72 ms per 2^20
+        // (1024-bit) and 3.29 -> 2.87 ms per 2^18 (2048-bit), but all-pairs cfg3
+        // 246.7 -> 256.0 ms and exact pairs 4.19 -> 4.38 ms, so only the RSA pairs
+        // kernel uses it.
+        if (ONE_ENTRY) {
+            if (resume == 1) goto roles_ba;
+        } else if (resume == 1) {
             if (hot(B, A, lB, tB, lA, tA)) {
                 resume = 0;
                 continue;
@@ -252,6 +260,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
                 resume = 1;
                 break;
             }
+        roles_ba:
             if (hot(B, A, lB, tB, lA, tA)) {
                 resume = 0;
                 break;
@@ -470,7 +479,7 @@ __global__ void BULKGCD_BOUNDS(W, true) pairs_kernel(PairsArgs a) {
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkRsa<W> sink{a.G, i, a.m_pad};
             NoPark np;
-            euclid_loop<W, STATS, false>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow, limbs,
+            euclid_loop<W, STATS, false, true>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow, limbs,
                                          slots, passw);
         } else {
             int k2 = 0;
@@ -488,7 +497,7 @@ __global__ void BULKGCD_BOUNDS(W, true) pairs_kernel(PairsArgs a) {
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkExact<W> sink{a.G, i, a.m_pad, k2, false, 0, 0};
             NoPark np;
-            euclid_loop<W, STATS, true>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, np, 0, iters, nslow, limbs, slots,
+            euclid_loop<W, STATS, true, false>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, np, 0, iters, nslow, limbs, slots,
                                         passw);
             // 64-bit tail: Case 1 of approx (lX <= 2): alpha = X div Y, exactly (L127).
             if (sink.tail) {
@@ -716,7 +725,7 @@ __global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
         unsigned K = pk.K;
         if (!allow_park) pk.K = 0;
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, pi, pj};
-        euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
+        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
                                      slots, passw);
         pk.K = K;
     };
@@ -754,11 +763,11 @@ __global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
         if (ParkCfg<W>::on) {
-            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
+            euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
                                          limbs, slots, passw);
         } else {
             NoPark np;
-            euclid_loop<W, STATS, false, RsaCond, HitSink<W>, NoPark>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
+            euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, NoPark>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
                                          limbs, slots, passw);
         }
         slot ^= 1;
