@@ -259,6 +259,21 @@ def test_pairs_config2_full_bit_exact(bg):
     assert int((oracle.bitlen_rows(G) > 1).sum()) >= 2  # the planted pairs are among them
 
 
+def test_pairs_config2_full_rsa_mode(bg):
+    """The RSA (early-terminate, L243-L255) pairs kernel on the full 2^20 pairs of
+    configs[1], the launch the one-entry resume of euclid_loop runs in: every result
+    equals the oracle's exact gcd when it has >= bits/2 bits, else 1 (reading 18)."""
+    A, B, ms = synth.config2()
+    G, _ = bg.bulkgcd_pairs_ex(A, B, 1024, bg.MODE_RSA)
+    Gx = oracle.gcd_batch(A, B)
+    hit = oracle.rsa_hit(oracle.bitlen_rows(Gx), 1024)
+    want = np.zeros_like(Gx)
+    want[:, 0] = 1
+    want[hit] = Gx[hit]
+    assert G.shape == want.shape and np.array_equal(G, want)
+    assert int(hit.sum()) >= 2  # the planted pairs are among them
+
+
 def test_pairs_chunked_host_path(bg):
     """Host batches above 2^18 pairs run in overlapped chunks on two streams:
     gcds and per-pair iteration counts equal single-chunk calls on the same
