@@ -86,8 +86,8 @@ def emit(W: int, form: str = "split", G: int = 1) -> str:
     outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(X[%d])' % k for k in range(W)]
     ins = ['"r"(Y[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)']
     o = ["template <>",
-         "__device__ __forceinline__ uint32_t duff_pass<%d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
-         "uint32_t alpha, int s, uint32_t &r) {" % (W, W, W),
+         "__device__ __forceinline__ uint32_t duff_pass<%d, %d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
+         "uint32_t alpha, int s, uint32_t &r) {" % (W, G, W, W),
          "  uint32_t zs;",
          '  asm volatile("%s"' % body,
          "      : %s" % ", ".join(outs),
@@ -169,8 +169,8 @@ def emit_two(W: int, G: int) -> str:
     outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(X[%d])' % k for k in range(W)]
     ins = ['"r"(Y[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)']
     o = ["template <>",
-         "__device__ __forceinline__ uint32_t duff_pass<%d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
-         "uint32_t alpha, int s, uint32_t &r) {" % (W, W, W),
+         "__device__ __forceinline__ uint32_t duff_pass<%d, %d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
+         "uint32_t alpha, int s, uint32_t &r) {" % (W, G, W, W),
          "  uint32_t zs;",
          '  asm volatile("%s"' % body,
          "      : %s" % ", ".join(outs),
@@ -186,6 +186,10 @@ def main():
     G = int(os.environ.get("BULKGCD_PASS_G", "4"))
     if form == "two":
         G = int(os.environ.get("BULKGCD_PASS_G", "8"))
+    # Exact-mode pairs kernel: G = 2 (cfg2 2^20 exact pairs 4.20 -> 3.87 ms; its larger
+    # code -- Case-1 tail, L41 normalisation -- misses the i-cache at G = 4).  G = 2 for
+    # the all-pairs kernel costs 246.7 -> 250.7 ms on cfg3, G = 8: 247.3 ms (exact 4.99).
+    GX = int(os.environ.get("BULKGCD_PASS_G_EXACT", "2"))
     here = os.path.dirname(os.path.abspath(__file__))
     parts = [
         "// GENERATED by gen_duff.py -- do not edit by hand.",
@@ -199,14 +203,19 @@ def main():
         "",
         "// Returns z_s (the lowest word of X - alpha*Y); r = ctz(z_s) (32 if z_s == 0, in which",
         "// case the funnel shifts wrap to 0 and X holds X - alpha*Y unshifted).",
-        "template <int W>",
+        "// G = limbs per straight-line block of the chain (one predicated branch per block).",
+        "template <int W, int G>",
         "__device__ __forceinline__ uint32_t duff_pass(uint32_t (&X)[W], const uint32_t (&Y)[W], uint32_t alpha, int s,",
         "                                              uint32_t &r);",
         "",
+        "constexpr int PASS_G = %d;        // all-pairs and RSA-mode pairs kernels" % G,
+        "constexpr int PASS_G_EXACT = %d;  // exact-mode pairs kernel (smaller code: i-cache)" % GX,
+        "",
     ]
     for W in WIDTHS:
-        parts.append(emit_two(W, G) if form == "two" else emit(W, form, G))
-        parts.append("")
+        for g in sorted({G, GX}):
+            parts.append(emit_two(W, g) if form == "two" else emit(W, form, g))
+            parts.append("")
     parts.append("}  // namespace bulkgcd")
     out = os.environ.get("BULKGCD_DUFF_OUT", os.path.join(here, "duff_pass.cuh"))
     with open(out, "w") as f:
