@@ -189,6 +189,7 @@ def main():
     # Exact-mode pairs kernel: G = 2 (cfg2 2^20 exact pairs 4.20 -> 3.87 ms; its larger
     # code -- Case-1 tail, L41 normalisation -- misses the i-cache at G = 4).  G = 2 for
     # the all-pairs kernel costs 246.7 -> 250.7 ms on cfg3, G = 8: 247.3 ms (exact 4.99).
+    # Exact at G = 1: 3.98 ms (2048-bit 3.74), G = 3: 4.00 ms (3.58), against 3.87 / 3.46 at G = 2.
     GX = int(os.environ.get("BULKGCD_PASS_G_EXACT", "2"))
     here = os.path.dirname(os.path.abspath(__file__))
     parts = [
