@@ -192,6 +192,7 @@ def main():
     # Exact at G = 1: 3.98 ms (2048-bit 3.74), G = 3: 4.00 ms (3.58), against 3.87 / 3.46 at G = 2.
     GX = int(os.environ.get("BULKGCD_PASS_G_EXACT", "2"))
     G64 = int(os.environ.get("BULKGCD_PASS_G", "2"))
+    G16 = int(os.environ.get("BULKGCD_PASS_G16", str(G)))  # W = 16 at G = 2: cfg6 82.6 -> 83.4 ms (stays 4)
     here = os.path.dirname(os.path.abspath(__file__))
     parts = [
         "// GENERATED by gen_duff.py -- do not edit by hand.",
@@ -213,12 +214,12 @@ def main():
         "// all-pairs and RSA-mode pairs kernels; W = 64 takes 2-limb blocks (cfg4 900.7 -> 898.4 ms,",
         "// 2^18 2048-bit RSA pairs 2.89 -> 2.81 ms; 8-limb blocks: 1,135 ms)",
         "template <int W>",
-        "constexpr int PASS_G = W >= 64 ? %d : %d;" % (G64, G),
+        "constexpr int PASS_G = W >= 64 ? %d : (W <= 16 ? %d : %d);" % (G64, G16, G),
         "constexpr int PASS_G_EXACT = %d;  // exact-mode pairs kernel (smaller code: i-cache)" % GX,
         "",
     ]
     for W in WIDTHS:
-        for g in sorted({G64 if W >= 64 else G, GX}):
+        for g in sorted({G64 if W >= 64 else (G16 if W <= 16 else G), GX}):
             parts.append(emit_two(W, g) if form == "two" else emit(W, form, g))
             parts.append("")
     parts.append("}  // namespace bulkgcd")
