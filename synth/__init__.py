@@ -14,7 +14,7 @@ top two bits set, so every n has exactly s bits):
 * modulus i is P[2i] * P[2i+1], P[t] = prime #t of the seed's stream;
 * a planted group G = (g0, g1, ...) replaces the first prime of every member
   after g0 with P[2*g0], so each pair inside G has gcd = P[2*g0] (the other
-  primes are distinct with overwhelming probability, checked by tests);
+  primes are distinct: primes_distinct(), asserted by tests for every config);
 * a duplicate (a, b) sets n_b = n_a, so gcd = n_a.
 
 Limbs are little-endian uint32, limb 0 least significant (include/bulkgcd.h).
@@ -180,6 +180,14 @@ def moduli(m: int, bits: int, seed: int, n_planted_pairs: int = 0, cliques=(), n
         truth.append((a, b, to_int(N[a])))
     truth.sort()
     return ModuliSet(bits, N, P, groups, dups, truth)
+
+
+def primes_distinct(ms: ModuliSet) -> bool:
+    """True iff every drawn prime of the set is distinct (sorting the rows of P).
+    With distinct primes the planted groups and duplicates are the only pairs that
+    share a factor, so ms.truth is the COMPLETE hit set."""
+    P = np.ascontiguousarray(ms.P)
+    return np.unique(P, axis=0).shape[0] == P.shape[0]
 
 
 # BASELINE.json configs[0..4] (SURVEY.md §8(d) M1).  Seed of config k is 2015 + k.

@@ -201,27 +201,35 @@ def test_all_pairs_stats_counters(bg, cfg1):
     assert int(ctr[4]) == sum(t.limb_steps for t in tr)      # limb-steps (the roofline's unit, M2)
 
 
-@pytest.mark.slow
+def _golden_hits(name):
+    """(sha256 of N, sorted [(i, j, g)]) from a tools/oracle_sweep.py golden file."""
+    import os
+    from conftest import GOLDEN
+    sha, hits = None, []
+    with open(os.path.join(GOLDEN, name)) as f:
+        for line in f:
+            if line.startswith("#"):
+                if "sha256(N) = " in line:
+                    sha = line.split("sha256(N) = ")[1].split()[0]
+                continue
+            i, j, g = line.split()
+            hits.append((int(i), int(j), int(g, 16)))
+    return sha, hits
+
+
 def test_all_pairs_config3_full(bg):
     """BASELINE configs[2] at full size, in the launch configuration bench.py times:
-    the exact hit set against construction ground truth, and a seeded sample of
-    pairs whose oracle gcd must then be < 2^(bits/2)."""
+    the GPU hit set equals, gcd by gcd, the full CPU-oracle sweep of all 134,209,536
+    pairs (tests/golden/cfg3_hits.txt, written by tools/oracle_sweep.py from oracle/
+    only), and equals the construction ground truth, which is complete because every
+    drawn prime is distinct."""
+    import hashlib
     ms = synth.config_moduli(3)
+    assert synth.primes_distinct(ms)
+    sha, golden = _golden_hits("cfg3_hits.txt")
+    assert sha == hashlib.sha256(np.ascontiguousarray(ms.N).tobytes()).hexdigest()
     hits = bg.bulkgcd_all_pairs(ms.N, 1024).as_list()
-    assert hits == ms.truth
-    rng = np.random.default_rng(3)
-    ii = rng.integers(0, ms.m, size=400_000)
-    jj = rng.integers(0, ms.m, size=400_000)
-    keep = ii < jj
-    ii, jj = ii[keep], jj[keep]
-    G = oracle.gcd_index_pairs(ms.N, ii, jj)
-    hit = oracle.rsa_hit(oracle.bitlen_rows(G), 1024)
-    truth = {(a, b) for a, b, _ in ms.truth}
-    for k in range(ii.size):
-        assert bool(hit[k]) == ((int(ii[k]), int(jj[k])) in truth)
-    # planted pairs through the oracle, gcd by gcd
-    for a, b, g in ms.truth:
-        assert oracle.gcd(synth.to_int(ms.N[a]), synth.to_int(ms.N[b])) == g
+    assert hits == golden == ms.truth
 
 
 def test_all_pairs_config4_full(bg):
@@ -229,6 +237,7 @@ def test_all_pairs_config4_full(bg):
     against construction ground truth, plus a seeded sample through the oracle."""
     ms = synth.config_moduli(4)
     assert ms.bits == 2048
+    assert synth.primes_distinct(ms)  # construction truth is the complete hit set (O5(f))
     hits = bg.bulkgcd_all_pairs(ms.N, 2048).as_list()
     assert hits == ms.truth
     rng = np.random.default_rng(4)
@@ -245,6 +254,7 @@ def test_all_pairs_config5_full(bg):
     """BASELINE configs[4] (65,536 moduli, 2,147,450,880 pairs) on one GPU: the
     exact hit set (33 planted pairs) against construction ground truth."""
     ms = synth.config_moduli(5)
+    assert synth.primes_distinct(ms)  # construction truth is the complete hit set (O5(f))
     hits = bg.bulkgcd_all_pairs(ms.N, 1024).as_list()
     assert len(ms.truth) == 33 and hits == ms.truth
 
@@ -342,3 +352,46 @@ def test_bench_multirank_path_gloo(bg):
     rec = json.loads(lines[0])
     assert rec["n_gpus"] == 2 and rec["config"]["hits_ok"] and rec["config"]["hits"] == 3
     assert rec["value"] > 0 and rec["e2e"]["value"] > 0
+
+
+def test_concurrent_host_threads(bg, cfg1):
+    """include/bulkgcd.h B5 (reentrant; the only global state is the lazily created
+    per-device context): 4 host threads call bulkgcd_pairs (one of them above the
+    2^18-pair chunk size, i.e. the two-stream chunked path) and bulkgcd_all_pairs at
+    the same time, three rounds each.  ctypes drops the GIL around the C calls, so the
+    calls overlap; every result must equal the oracle's."""
+    import threading
+    jobs = []
+    for t in range(4):
+        if t == 0:
+            A, B, _ = synth.config2(300_000)
+        else:
+            a, b = synth.mixed_pairs(2000 + 500 * t, 1024, seed=700 + t)
+            A, B = synth.from_ints(a, 32), synth.from_ints(b, 32)
+        ms = synth.moduli(96 + 32 * t, 1024, seed=800 + t, n_planted_pairs=2, cliques=(3,))
+        jobs.append((A, B, ms))
+    out = [[] for _ in jobs]
+    errs = []
+
+    def work(t):
+        try:
+            A, B, ms = jobs[t]
+            for _ in range(3):
+                out[t].append((bg.bulkgcd_pairs(A, B, 1024), bg.bulkgcd_all_pairs(ms.N, 1024).as_list()))
+        except Exception as e:  # noqa: BLE001 -- reported below
+            errs.append((t, repr(e)))
+
+    th = [threading.Thread(target=work, args=(t,)) for t in range(len(jobs))]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join()
+    assert not errs, errs
+    for (A, B, ms), res in zip(jobs, out):
+        want_g = oracle.gcd_batch(A, B)
+        want_h = oracle.all_pairs_hits(ms.N, 1024)
+        assert want_h == ms.truth
+        assert len(res) == 3
+        for G, hits in res:
+            assert np.array_equal(G, want_g)
+            assert hits == want_h

@@ -91,12 +91,12 @@ def test_pairs_4096_iteration_parity(bg, ms4096):
 
 def test_table4_4096_means(bg):
     """Table IV column (E) at 4096 bits from the GPU's per-pair
-    iteration counts over 2000 pairs.  The printed 4096 rows are swapped (DESIGN.md
-    reading 19): non-terminate 1523.2, early-terminate 761.6.  Inputs: seeded odd
+    iteration counts over 2000 pairs (the golden file stores the 4096 rows de-garbled,
+    DESIGN.md reading 19: non-terminate 1523.2, early-terminate 761.6).  Inputs: seeded odd
     4096-bit integers with the top two bits set (the size statistics of RSA moduli;
     generating 4000 2048-bit primes would take minutes)."""
     tab = {(r[0], int(r[1])): [float(x) for x in r[2:]] for r in read_golden("table4_iterations.txt")}
-    nonterm_paper, early_paper = tab[("early", 4096)][4], tab[("nonterm", 4096)][4]
+    nonterm_paper, early_paper = tab[("nonterm", 4096)][4], tab[("early", 4096)][4]
     rng = np.random.default_rng(6001)
     X = rng.integers(0, 1 << 32, size=(4000, 128), dtype=np.uint64).astype(np.uint32)
     X[:, 0] |= 1

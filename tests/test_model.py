@@ -156,12 +156,14 @@ def test_table4_binary_columns(bits, npairs):
     N = synth.ints(ms.N)
     for col, fn in ((2, am.binary_euclid), (3, am.fast_binary_euclid)):
         for mode, early in (("early", bits), ("nonterm", None)):
-            arr = np.array([fn(N[k], N[k + 1], early).iterations for k in range(npairs)], float)
+            # (C) early-terminate has no listing in the paper (only (E)'s, L255).  Its printed means
+            # (L303/L305) fit a threshold of s/2 - 1 bits, not (E)'s s/2 (reading 20: with
+            # s/2 our mean sits 1.5 iterations = 11 standard errors low at 512 bits).  The model is
+            # pinned here under that reading; the GPU kernels keep (E)'s s/2 for every algorithm.
+            kw = {"early_offset": 1} if (col, mode) == (2, "early") else {}
+            arr = np.array([fn(N[k], N[k + 1], early, **kw).iterations for k in range(npairs)], float)
             paper = tab[(mode, bits)][col]
             se = math.sqrt(arr.var() / arr.size + arr.var() / 10000)
-            # (C) early-terminate: the paper gives no listing, only (E)'s (L255); with (E)'s loop-head
-            # test our mean is 0.2-0.5% below the printed one (reading 20): checked to 0.6%.
-            tol = 0.006 * paper if (col, mode) == (2, "early") else 3 * se + 0.05
-            assert abs(arr.mean() - paper) <= tol, (col, mode, bits, arr.mean(), paper, se)
+            assert abs(arr.mean() - paper) <= 3 * se + 0.05, (col, mode, bits, arr.mean(), paper, se)
     g = [am.binary_euclid(N[k], N[k + 1]).gcd for k in range(50)]
     assert g == [math.gcd(N[k], N[k + 1]) for k in range(50)]

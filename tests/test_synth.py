@@ -47,3 +47,14 @@ def test_config2_pairs():
     i, j = synth.pair_indices(synth.CFG2_POOL, synth.CFG2_PAIRS)
     assert i.size == 1 << 20 and np.all(i < j)
     assert (int(i[0]), int(j[0])) == (0, 1)
+
+
+def test_config_primes_distinct_small():
+    """Every drawn prime of configs[0] and of the cfg2 pool is distinct, so their
+    construction truth is complete; cfg3/4/5 are asserted
+    by the GPU full-size tests, which generate those sets anyway."""
+    assert synth.primes_distinct(synth.config_moduli(1))
+    _, _, pool = synth.config2(16)
+    assert pool.P.shape == (2 * synth.CFG2_POOL, 16) and synth.primes_distinct(pool)
+    bad = synth.ModuliSet(1024, pool.N[:2], np.concatenate([pool.P[:3], pool.P[:1]]))
+    assert not synth.primes_distinct(bad)
