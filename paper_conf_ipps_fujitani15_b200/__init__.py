@@ -39,6 +39,24 @@ SYMBOLS = (
 )
 
 
+def check_moduli(N: np.ndarray, bits: int) -> None:
+    """The host API's RSA-mode input rule (include/bulkgcd.h B2; PAPER.md L41 assumes odd
+    inputs): every modulus odd and > 1, shape [n, bits/32].  bulkgcd_all_pairs_band
+    does not check it on the device, so the band drivers (dist.py, resume.py) do:
+    a zero modulus would be reported against every other one, an even one would lose
+    its factors of 2."""
+    W = bits // 32
+    if N.ndim != 2 or N.shape[1] != W:
+        raise ValueError(f"moduli must be uint32[n, {W}] for {bits} bits, got shape {N.shape}")
+    if N.shape[0] == 0:
+        return
+    odd = (N[:, 0] & 1) == 1
+    gt1 = (N[:, 0] > 1) | np.any(N[:, 1:] != 0, axis=1)
+    bad = np.nonzero(~(odd & gt1))[0]
+    if bad.size:
+        raise ValueError(f"modulus {int(bad[0])} is even or <= 1 (RSA mode needs odd moduli > 1)")
+
+
 class BulkGcdError(RuntimeError):
     def __init__(self, code: int, msg: str):
         super().__init__(f"libbulkgcd error {code}: {msg}")

@@ -10,6 +10,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <numeric>
 #include <vector>
 
@@ -50,6 +51,25 @@ int words_for(uint32_t bits) {
     }
 }
 
+// Per-device one-time set-up (B5: the only global state is a lazily created per-device
+// context).  One instance per call site: `run` executes f() once per device, under a
+// mutex, and only records success -- a failed attempt is retried by the next call.
+// Thread-safe; a process that drives several GPUs gets the set-up on every device.
+struct PerDeviceOnce {
+    std::mutex mu;
+    bool done[64] = {};
+    template <class F>
+    int run(F f) {
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return f();
+        std::lock_guard<std::mutex> lock(mu);
+        if (done[dev]) return 0;
+        int rc = f();
+        if (rc == 0) done[dev] = true;
+        return rc;
+    }
+};
+
 int sm_count() {
     int dev = 0, n = 148;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
@@ -70,16 +90,15 @@ int device_check() {
     // default the pool unmaps everything at each synchronisation, so a repeated call
     // re-maps its buffers (hundreds of MB for bulkgcd_pairs).  Keep up to 4 GiB cached
     // in the device's default pool (the per-device context of include/bulkgcd.h B5).
-    static bool pool_set[64] = {};  // idempotent, benign race
-    if (dev < 64 && !pool_set[dev]) {
+    static PerDeviceOnce pool_once;
+    return pool_once.run([&]() -> int {
         cudaMemPool_t pool;
         if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
             uint64_t keep = 4ull << 30;
             cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
         }
-        pool_set[dev] = true;
-    }
-    return 0;
+        return 0;
+    });
 }
 
 // RAII stream-ordered device buffer.
@@ -106,14 +125,15 @@ size_t pad32(size_t m) { return (m + 31) / 32 * 32; }
 template <int W, int ALG>
 int launch_pairs_smem_alg(const PairsArgs &a, int mode, bool stats, cudaStream_t st) {
     constexpr size_t smem = smem_operand_bytes<W>();
-    static bool attr_done = false;  // idempotent, benign race
-    if (!attr_done) {
-        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        attr_done = true;
-    }
+    static PerDeviceOnce attr_once;  // dynamic shared memory opt-in, per device
+    if (int rc = attr_once.run([]() -> int {
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            return 0;
+        }))
+        return rc;
     uint64_t cohorts = (a.m + 31) / 32;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * smem_blocks<W>(), (cohorts + 1) / 2);
     if (grid == 0) return 0;
@@ -166,12 +186,13 @@ int launch_pairs(const uint32_t *dA, const uint32_t *dB, uint32_t *dG, size_t m,
 template <int W, int ALG>
 int launch_allpairs_smem_alg(const AllPairsArgs &a, bool stats, cudaStream_t st) {
     constexpr size_t smem = smem_operand_bytes<W>();
-    static bool attr_done = false;  // idempotent, benign race
-    if (!attr_done) {
-        CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        attr_done = true;
-    }
+    static PerDeviceOnce attr_once;  // dynamic shared memory opt-in, per device
+    if (int rc = attr_once.run([]() -> int {
+            CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            return 0;
+        }))
+        return rc;
     uint64_t warps = a.c_end - a.c_begin;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * smem_blocks<W>(), (warps + 1) / 2);
     if (stats) allpairs_smem_kernel<W, true, ALG><<<(unsigned)grid, SM_THREADS, smem, st>>>(a);
@@ -211,12 +232,13 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
         a.park = park.p;
     }
     constexpr size_t smem = allpairs_smem_bytes<W>();
-    static bool attr_done[2] = {false, false};  // idempotent, benign race
-    if (!attr_done[0]) {
-        CK(cudaFuncSetAttribute(allpairs_kernel<W, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(allpairs_kernel<W, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        attr_done[0] = true;
-    }
+    static PerDeviceOnce attr_once;  // dynamic shared memory opt-in, per device
+    if (int rc = attr_once.run([]() -> int {
+            CK(cudaFuncSetAttribute(allpairs_kernel<W, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(allpairs_kernel<W, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            return 0;
+        }))
+        return rc;
     if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
     else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, smem, st>>>(a);
     CK(cudaGetLastError());
@@ -328,9 +350,14 @@ int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t 
 // with pageable ones the driver stages the copies synchronously and the result is the same.
 constexpr size_t PAIRS_CHUNK = size_t(1) << 18;
 
+// Scope guard of the chunked path: on every exit -- including an error return in the
+// middle of the chunk loop -- both streams are drained before they are destroyed, so no
+// copy into the caller's G / iters is still in flight when the call returns.
 struct StreamPair {
     cudaStream_t s[2] = {nullptr, nullptr};
     ~StreamPair() {
+        for (auto &x : s)
+            if (x) cudaStreamSynchronize(x);
         for (auto &x : s)
             if (x) cudaStreamDestroy(x);
     }

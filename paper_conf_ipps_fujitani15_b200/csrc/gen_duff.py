@@ -180,6 +180,70 @@ def emit_two(W: int, G: int) -> str:
     return "\n".join(o)
 
 
+def emit_cmpl(W: int, G: int, ones: bool) -> str:
+    """Complement form (round 2): one operand of the pair is kept bit-complemented, so
+    the update is a pure multiply-accumulate  T = X + alpha*Y + cin  (mod D^n, n = W - s)
+    and the subtract-with-borrow chain of the split form disappears:
+      * A-type (ones=True): X holds ~X0, Y plain, cin = 0:  T = D^n - 1 - (X0 - alpha*Y),
+        so the complemented result is T >> r with ones shifted in at the top, r = ctz(~t_s);
+      * B-type (ones=False): X plain, Y holds ~Y0, cin = alpha:  T = X - alpha*Y0 (mod D^n,
+        exact since 0 <= X - alpha*Y0 < D^n), zeros shifted in, r = ctz(t_s).
+    Per limb t_k + D c_k = alpha*y_k + x_k + c_{k-1} < 2^64, written as one 64-bit
+    mad.wide plus one 64-bit add, which ptxas lowers to IMAD.WIDE.U32 + a three-input
+    IADD3 (two carry-outs) + IADD3.X (two carry-ins): 4 instructions per limb with the
+    funnel shift, against 5 for the split form (tools/limbmix2.cu: 8.8 vs 9.5 SMSP-cycles).
+
+    Operands: %0 = r (out), %1 = t_s (out), %2..%(W+1) = X[k] (in/out),
+    %(W+2)..%(2W+1) = Y[k], %(2W+2) = alpha, %(2W+3) = s, %(2W+4) = cin."""
+    xa = lambda k: "%%%d" % (2 + k)
+    ya = lambda k: "%%%d" % (W + 2 + k)
+    al = "%%%d" % (2 * W + 2)
+    sa = "%%%d" % (2 * W + 3)
+    ci = "%%%d" % (2 * W + 4)
+    a = ["{", ".reg .u32 tp, t, c, u;", ".reg .u64 p, q, w;", ".reg .pred pe;",
+         "setp.ge.s32 pe, %s, 0;" % sa,
+         "ts: .branchtargets %s;" % ", ".join("E%d" % k for k in range(W)),
+         "brx.idx %s, ts;" % sa]
+
+    def mac(k, cin, dst):
+        return ["cvt.u64.u32 q, %s;" % xa(k),
+                "mad.wide.u32 p, %s, %s, q;" % (al, ya(k)),
+                "cvt.u64.u32 w, %s;" % cin,
+                "add.u64 p, p, w;",
+                "mov.b64 {%s, c}, p;" % dst]
+
+    def limb(k):
+        return mac(k, "c", "t") + ["shf.r.wrap.b32 %s, tp, t, %%0;" % xa(k - 1), "mov.u32 tp, t;"]
+
+    for k in range(W):
+        e = min((k // G + 1) * G, W)
+        nxt = "B%d" % e if e < W else "TOP"
+        a += ["E%d:" % k] + mac(k, ci, "tp") + ["mov.u32 %1, tp;"]
+        a += (["not.b32 u, tp;", "brev.b32 u, u;"] if ones else ["brev.b32 u, tp;"]) + ["clz.b32 %0, u;"]
+        for j in range(k + 1, e):
+            a += limb(j)
+        a.append("@pe bra %s;" % nxt)
+    a.append("bra.uni TOP;")
+    for k in range(1, W):
+        if k % G == 0:
+            a.append("B%d:" % k)
+        a += limb(k)
+    a += ["TOP:", "shf.r.wrap.b32 %s, tp, %s, %%0;" % (xa(W - 1), "0xffffffff" if ones else "0"), "}"]
+    body = "\\n\\t".join(x.replace('"', '\\"') for x in a)
+    outs = ['"=r"(r)', '"=r"(ts)'] + ['"+r"(X[%d])' % k for k in range(W)]
+    ins = ['"r"(Y[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)', '"r"(cin)']
+    o = ["template <>",
+         "__device__ __forceinline__ uint32_t duff_cpass<%d, %d, %s>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
+         "uint32_t alpha, uint32_t cin, int s, uint32_t &r) {" % (W, G, "true" if ones else "false", W, W),
+         "  uint32_t ts;",
+         '  asm volatile("%s"' % body,
+         "      : %s" % ", ".join(outs),
+         "      : %s);" % ", ".join(ins),
+         "  return ts;",
+         "}"]
+    return "\n".join(o)
+
+
 def main():
     import sys
     form = sys.argv[1] if len(sys.argv) > 1 else os.environ.get("BULKGCD_PASS_FORM", "split")
@@ -191,7 +255,7 @@ def main():
     # the all-pairs kernel costs 246.7 -> 250.7 ms on cfg3, G = 8: 247.3 ms (exact 4.99).
     # Exact at G = 1: 3.98 ms (2048-bit 3.74), G = 3: 4.00 ms (3.58), against 3.87 / 3.46 at G = 2.
     GX = int(os.environ.get("BULKGCD_PASS_G_EXACT", "2"))
-    G64 = int(os.environ.get("BULKGCD_PASS_G", "2"))
+    G64 = int(os.environ.get("BULKGCD_PASS_G64", "2"))  # W = 64 has its own knob
     G16 = int(os.environ.get("BULKGCD_PASS_G16", str(G)))  # W = 16 at G = 2: cfg6 82.6 -> 83.4 ms (stays 4)
     here = os.path.dirname(os.path.abspath(__file__))
     parts = [
@@ -218,9 +282,21 @@ def main():
         "constexpr int PASS_G_EXACT = %d;  // exact-mode pairs kernel (smaller code: i-cache)" % GX,
         "",
     ]
+    parts += [
+        "// Complement form (emit_cmpl): T = X + alpha*Y + cin (mod D^n); ONES: shift ones in at the",
+        "// top and r = ctz(~t_s) (X holds a complemented operand).  Returns t_s.",
+        "template <int W, int G, bool ONES>",
+        "__device__ __forceinline__ uint32_t duff_cpass(uint32_t (&X)[W], const uint32_t (&Y)[W], uint32_t alpha,",
+        "                                               uint32_t cin, int s, uint32_t &r);",
+        "",
+    ]
     for W in WIDTHS:
-        for g in sorted({G64 if W >= 64 else (G16 if W <= 16 else G), GX}):
+        gw = G64 if W >= 64 else (G16 if W <= 16 else G)
+        for g in sorted({gw, GX}):
             parts.append(emit_two(W, g) if form == "two" else emit(W, form, g))
+            parts.append("")
+        for ones in (True, False):
+            parts.append(emit_cmpl(W, gw, ones))
             parts.append("")
     parts.append("}  // namespace bulkgcd")
     out = os.environ.get("BULKGCD_DUFF_OUT", os.path.join(here, "duff_pass.cuh"))

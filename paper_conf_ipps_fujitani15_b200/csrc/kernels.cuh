@@ -3,6 +3,7 @@
 // (bulkgcd_all_pairs / bulkgcd_all_pairs_band).
 #pragma once
 #include <cstdint>
+#include <type_traits>
 
 #include "euclid.cuh"
 #include "smem_euclid.cuh"
@@ -158,28 +159,45 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // Sink API: quick(fin, lX, tX, lY, tY) runs in the hot loop for every lane
 // and returns true if a finished lane needs cold(...) (warp-converged, with
 // the operand registers); scalar-only finishes are handled by quick itself.
-template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, class Parker>
+//
+// CMPL: complement form (gen_duff.py emit_cmpl) -- A is kept bit-complemented in its
+// registers for the whole loop and B plain, so every update is a multiply-accumulate:
+// hot(A, B) runs the A-type pass (A~ + alpha*B, ones shifted in), hot(B, A) the B-type
+// pass (B + alpha*A~ + alpha).  The roles alternate strictly, which keeps A complemented;
+// the rare cold-section code that reads the operand registers (fix-ups, the hit sink)
+// sees plain values (A is complemented around it).
+template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, class Parker, bool CMPL = false>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, Parker &pk, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
                                             uint32_t &passw) {
+    static_assert(!(CMPL && Parker::enabled), "complement form: no straggler parking");
+    using CmA = std::integral_constant<int, CMPL ? 1 : 0>;  // hot_iter pass form with A updated
+    using CmB = std::integral_constant<int, CMPL ? 2 : 0>;  // ... with B updated
     int s = s0;
     int fix = 0;     // pending fix-up of the last iteration (hot_iter's code)
     int resume = 0;  // roles of the next iteration: 0 -> (X, Y) = (A, B), 1 -> (B, A)
+    if (CMPL) cmpl_regs<W>(A);
 
     // Cold section for the next roles (X, Y); the last iteration ran on (Y, X).
     // Applies fix-ups, runs the loop test, serves finished lanes, realigns.
     auto cold = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
         if (__any_sync(FULL, fix != 0)) {
             if (STATS && fix >= 2) ++nslow;
+            if (CMPL) cmpl_regs<W>(A);
             apply_fix<W>(fix, Y, X, lY, tY, lX, tX, s);
+            if (CMPL) cmpl_regs<W>(A);
             fix = 0;
         }
         bool run = live & cond(lX, tX, lY, tY);
         bool fin = live & !run;
         if (__any_sync(FULL, fin)) {
             bool need = sink.quick(fin, lX, tX, lY, tY);
-            if (__any_sync(FULL, need)) sink.cold(need, X, Y, lX, tX, lY, tY, s);
+            if (__any_sync(FULL, need)) {
+                if (CMPL) cmpl_regs<W>(A);
+                sink.cold(need, X, Y, lX, tX, lY, tY, s);
+                if (CMPL) cmpl_regs<W>(A);
+            }
         }
         live = run;
         unsigned brun = __ballot_sync(FULL, run);
@@ -200,7 +218,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
     // One hot iteration on roles (X, Y) (its loop test already passed: the
     // live lanes are the running ones), then the loop test of the next
     // iteration (roles (Y, X)).  Returns true to go cold.
-    auto hot = [&](uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
+    auto hot = [&](auto cm, uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
         if (STATS) {
             ++slots;
             passw += W - s;  // words the warp's pass covers this iteration
@@ -210,7 +228,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
             }
         }
         bool full, post, lt;
-        hot_iter<W, EXACT>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
+        hot_iter<W, EXACT, decltype(cm)::value>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
         bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
         bool fin = live & !run & !bad;
@@ -250,18 +268,18 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         if (ONE_ENTRY) {
             if (resume == 1) goto roles_ba;
         } else if (resume == 1) {
-            if (hot(B, A, lB, tB, lA, tA)) {
+            if (hot(CmB{}, B, A, lB, tB, lA, tA)) {
                 resume = 0;
                 continue;
             }
         }
         for (;;) {
-            if (hot(A, B, lA, tA, lB, tB)) {
+            if (hot(CmA{}, A, B, lA, tA, lB, tB)) {
                 resume = 1;
                 break;
             }
         roles_ba:
-            if (hot(B, A, lB, tB, lA, tA)) {
+            if (hot(CmB{}, B, A, lB, tB, lA, tA)) {
                 resume = 0;
                 break;
             }
@@ -665,6 +683,15 @@ __device__ __forceinline__ void cohort_coords(uint64_t c, uint64_t n, uint64_t &
     j = 32 * b + 1 + (c - cohorts_before(b, n));
 }
 
+// Complement-form pass (gen_duff.py emit_cmpl) in the all-pairs kernel, by width:
+// measured on B200, cfg4 (2048-bit) 899.7 -> 852.1 ms, but cfg3 (1024-bit) 246.8 -> 255.1 ms
+// and cfg6 (512-bit) 82.6 -> 83.9 ms (more spills at 96 / 64 registers): W = 64 only.
+#ifndef BULKGCD_ALLPAIRS_CMPL_MIN_W
+#define BULKGCD_ALLPAIRS_CMPL_MIN_W 64
+#endif
+template <int W>
+__host__ __device__ constexpr bool allpairs_cmpl() { return W >= BULKGCD_ALLPAIRS_CMPL_MIN_W; }
+
 template <int W, bool STATS>
 __global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -767,8 +794,8 @@ __global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
                                          limbs, slots, passw);
         } else {
             NoPark np;
-            euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, NoPark>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow,
-                                         limbs, slots, passw);
+            euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, NoPark, allpairs_cmpl<W>()>(
+                A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow, limbs, slots, passw);
         }
         slot ^= 1;
         have = have2;

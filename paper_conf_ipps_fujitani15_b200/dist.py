@@ -18,7 +18,7 @@ import torch
 import torch.distributed as dist
 
 from . import (FLAG_STATS, Hits, bulkgcd_all_pairs_band, bulkgcd_blocked_words, bulkgcd_cohort_count,
-               bulkgcd_layout_blocked)
+               bulkgcd_layout_blocked, check_moduli)
 
 
 def band(total: int, world: int, rank: int) -> tuple[int, int]:
@@ -36,6 +36,7 @@ class AllPairsBand:
         self.n = int(N.shape[0])
         self.device = torch.device(device if device is not None else "cuda")
         N = np.ascontiguousarray(N, dtype=np.uint32)
+        check_moduli(N, bits)
         self.h_N = torch.from_numpy(N.view(np.int32)).pin_memory() if self.device.type == "cuda" else \
             torch.from_numpy(N.view(np.int32))
         self.d_N = torch.empty(self.h_N.shape, dtype=torch.int32, device=self.device)

@@ -31,7 +31,7 @@ from dataclasses import dataclass
 
 import numpy as np
 
-from . import Hits, bulkgcd_cohort_count
+from . import Hits, bulkgcd_cohort_count, check_moduli
 
 FORMAT = "bulkgcd-resume-v1"
 
@@ -120,8 +120,7 @@ def all_pairs_resumable(N: np.ndarray, bits: int, checkpoint: str, *, chunk: int
         raise ValueError("chunk must be >= 1")
     N = np.ascontiguousarray(N, dtype=np.uint32)
     W = bits // 32
-    if N.ndim != 2 or N.shape[1] != W:
-        raise ValueError(f"expected uint32[n, {W}] moduli")
+    check_moduli(N, bits)
     n = int(N.shape[0])
     c_begin, c_end = part_range(bulkgcd_cohort_count(n), parts, part)
     want = State(n, bits, digest(N), c_begin, c_end, c_begin, np.zeros((0, 2 + W), np.uint32))
