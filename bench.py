@@ -65,6 +65,7 @@ WORKLOADS = {
 UNIT = "GCD/s"
 OPS_PER_LIMB, OPS_PER_ITER = 4, 16  # SURVEY.md §8(d) M2; DESIGN.md §Roofline
 ALU_OPS_PER_LIMB = 3  # of the 4: IADD3, IADD3.X, SHF.R.W (ALU pipe); IMAD.WIDE.U32 is on the FMA pipe
+PAPER_E_US = {512: 9.40, 1024: 28.6, 2048: 96.4, 4096: 357.0}  # Table V CPU (E), early-terminate, Xeon X7460 (L485-L493)
 
 
 BACKEND = os.environ.get("BULKGCD_BENCH_BACKEND", "nccl")  # "gloo": test mode, ranks may share one GPU
@@ -101,58 +102,65 @@ def _peaks():
         return {"sm_max_mhz": 1965.0}, "fallback"
 
 
-def _pipe_rates():
-    """Measured sm_100a issue rates on this pool's B200s (tools/pipemix.cu,
-    profiles/r1_pipemix.json), warp-instructions/clk/SM: the ALU pipe (SHF.R.W
-    alone, the pipe IADD3 carry chains and SHF share) and the best two-pipe mix
-    (the integer issue ceiling)."""
+def _alu_rate():
+    """Measured ALU-pipe issue rate on this pool's B200s, warp-instructions/clk/SM:
+    SHF.R.W alone (tools/pipemix.cu -> profiles/r1_pipemix.json; tools/pipemix2.cu
+    -> profiles/r2_pipemix2.json re-measures 2.04 SMSP-cycles per SHF = 1.96/clk/SM)."""
     try:
         with open(os.path.join(ROOT, "profiles", "r1_pipemix.json")) as f:
-            r = json.load(f)["rates"]
-        return float(r["SHF"]), max(float(r["SHF+IMAD"]), float(r["SEL+IMAD"]))
+            return float(json.load(f)["rates"]["SHF"]), "measured (profiles/r1_pipemix.json, SHF.R.W alone)"
     except (OSError, ValueError, KeyError):
-        return None, None
+        return 2.0, "guide unit counts (16 ALU lanes per SMSP)"
 
 
-def roofline(limbs, iters, n_gcd, kern_s, sms, kernel, share, traffic):
-    """Roofline of the Euclid kernel.  Bound: the ALU pipe (ncu: the
-    busiest unit, profiles/).  Algorithmic ALU-pipe work = 3 lane-ops per limb-step
-    (IADD3 carry-add, IADD3.X borrow, SHF.R.W funnel: the minimal sm_100a limb; its
-    IMAD.WIDE.U32 runs on the FMA pipe in parallel) + 16 per iteration (SURVEY.md
-    §8(d) M2), counted exactly by the kernel's stats pass, over the kernel's
-    CUDA-event time, against the measured ALU-pipe rate x 32 lanes x SMs x the max
-    SM clock (MEASURED_PEAKS.json; NVML shows it held under load).  Also reported:
-    all 4 + 16 ops against the measured integer issue ceiling and the guide's
-    4 warp-instructions/clk/SM."""
+# SURVEY.md §8(d) M2: ops_alg = 4 L + 16 I.  Of the 4 per limb-step, 3 are ALU-pipe (IADD3 / IADD3.X
+# carry chains and the SHF.R.W funnel) and 1 (IMAD.WIDE.U32) FMA-heavy; of the 16 per iteration we
+# count 8 as ALU-pipe (top-word fetch 2, compare 2, alpha select / parity 2, vote + branch 2) and 8
+# as FP64 / XU / FMA work (reciprocal seed, Newton steps, quotient, conversions) -- DESIGN.md §7.
+ALU_OPS_PER_ITER = 8
+
+
+def roofline(limbs, iters, n_gcd, kern_s, sms, kernel, share, traffic, eff=None):
+    """Roofline of the Euclid kernel.
+
+    Bound "alu": integer issue.  achieved = algorithmic integer lane-ops per launch,
+    ops_alg = 4 L + 16 I (M2; L = limb-steps, I = iterations, counted exactly by the
+    kernel's stats pass on the same input), over the kernel's CUDA-event duration;
+    peak P_int = SMs x 4 SMSPs x 32 lanes x 1 instruction/clk x the max SM clock
+    (MEASURED_PEAKS.json sm_max_mhz; the guide's dispatch width: MEASURED_PEAKS has
+    no integer peak).  Secondary "alu_pipe": the ALU-pipe share of ops_alg
+    (3 L + 8 I) against the measured ALU-pipe rate.  `eff`: SIMT efficiencies from
+    the stats pass (lane = useful lane-iterations / lane-slots; pass-word = limb-steps
+    / words the warp's passes covered)."""
     peaks, src = _peaks()
     f = float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
-    alu_ipc, issue_ipc = _pipe_rates()
-    src_alu = "measured (profiles/r1_pipemix.json)"
-    if alu_ipc is None:
-        alu_ipc, issue_ipc, src_alu = 2.0, 4.0, "guide unit counts (no pipemix measurement)"
-    alu_ops = (ALU_OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / kern_s
-    all_ops = (OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / kern_s
-    peak = sms * 32 * alu_ipc * f
-    issue_peak = sms * 32 * issue_ipc * f
-    guide = sms * 128 * f
-    return {"bound": "alu", "achieved": alu_ops / 1e12, "peak": peak / 1e12, "unit": "T ALU-pipe lane-ops/s",
-            "frac": alu_ops / peak, "traffic": traffic, "kernel": kernel, "kernel_ms": kern_s * 1e3,
-            "kernel_share_of_step": share,
-            "alu_ops_per_gcd": (ALU_OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / n_gcd,
-            "ops_per_gcd": (OPS_PER_LIMB * limbs + OPS_PER_ITER * iters) / n_gcd,
-            "peak_source": (f"ALU pipe {alu_ipc:.3f} warp-instr/clk/SM ({src_alu}) x 32 lanes x {sms} SMs x "
-                            f"{f / 1e6:.0f} MHz ({src} MEASURED_PEAKS sm_max_mhz)"),
-            "issue": {"achieved": all_ops / 1e12, "peak": issue_peak / 1e12, "frac": all_ops / issue_peak,
-                      "unit": "T int lane-ops/s", "ipc": issue_ipc},
-            "peak_guide": guide / 1e12, "frac_of_guide_peak": all_ops / guide}
+    alu_ipc, alu_src = _alu_rate()
+    ops = OPS_PER_LIMB * limbs + OPS_PER_ITER * iters
+    alu_ops = ALU_OPS_PER_LIMB * limbs + ALU_OPS_PER_ITER * iters
+    p_int = sms * 4 * 32 * f
+    p_alu = sms * 32 * alu_ipc * f
+    out = {"bound": "alu", "achieved": ops / kern_s / 1e12, "peak": p_int / 1e12, "unit": "T int lane-ops/s",
+           "frac": ops / kern_s / p_int, "traffic": traffic, "kernel": kernel, "kernel_ms": kern_s * 1e3,
+           "kernel_share_of_step": share, "ops_per_gcd": ops / n_gcd,
+           "limb_steps_per_gcd": limbs / n_gcd, "iterations_per_gcd": iters / n_gcd,
+           "peak_source": (f"P_int = {sms} SMs x 4 SMSPs x 32 lanes x 1 warp-instr/clk x {f / 1e6:.0f} MHz "
+                           f"({src} MEASURED_PEAKS sm_max_mhz; SURVEY.md §8(d) M3, guide dispatch width)"),
+           "alu_pipe": {"achieved": alu_ops / kern_s / 1e12, "peak": p_alu / 1e12, "frac": alu_ops / kern_s / p_alu,
+                        "unit": "T ALU-pipe lane-ops/s", "ops_per_gcd": alu_ops / n_gcd,
+                        "peak_source": f"ALU pipe {alu_ipc:.3f} warp-instr/clk/SM ({alu_src}) x 32 x {sms} x "
+                                       f"{f / 1e6:.0f} MHz"}}
+    if eff:
+        out.update(eff)
+    return out
 
 
-def _traffic():
-    """dram bytes per launch of the all-pairs kernel from the committed ncu summary."""
+def _traffic(workload: str):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch of the workload's hot kernel,
+    from the committed ncu --set full summary of the current build
+    (profiles/r2_ncu_traffic.json, written by tools/ncu_traffic.py); None if absent."""
     try:
-        with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as f:
-            s = json.load(f)
-        return s.get("allpairs_dram_bytes_per_launch")
+        with open(os.path.join(ROOT, "profiles", "r2_ncu_traffic.json")) as f:
+            return json.load(f).get(workload, {}).get("dram_bytes_per_launch")
     except (OSError, ValueError):
         return None
 
@@ -207,36 +215,56 @@ class ClockSampler:
                 "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def cpu_baseline(ms, target_s: float = 12.0, seed: int = 7):
-    """The oracle (oracle/gcd_oracle.c, as it stands) on a bounded sample of the
-    workload's pairs, all host cores.  Returns the cpu_baseline object."""
+REF_CALL_PAIRS = 1 << 18  # pairs per oracle call, shared by cpu_baseline and the --impl reference arm
+
+
+def _sample_pairs(rng, m: int, k: int):
+    """k seeded random pairs (i < j) of an m-moduli all-pairs workload."""
+    i = rng.integers(0, m, size=2 * k + 64)
+    j = rng.integers(0, m, size=2 * k + 64)
+    keep = i < j
+    return i[keep][:k], j[keep][:k]
+
+
+def cpu_baseline(ms, target_s: float = 10.0, seed: int = 7):
+    """The oracle (oracle/gcd_oracle.c, as it stands: classical Euclid + Knuth D) on a
+    bounded seeded sample of the workload's pairs, all host cores, in calls of
+    REF_CALL_PAIRS pairs (the reference arm's step), plus two single-core figures: the
+    oracle, and the paper's own algorithm in C (oracle/approx_euclid.c, early-terminate:
+    the analogue of Table V's CPU (E) column)."""
     import oracle
     cores = os.cpu_count() or 1
     rng = np.random.default_rng(seed)
-
-    def sample(k):
-        i = rng.integers(0, ms.m, size=2 * k)
-        j = rng.integers(0, ms.m, size=2 * k)
-        keep = i < j
-        return i[keep][:k], j[keep][:k]
-
-    i, j = sample(1 << 14)  # calibration
-    t0 = time.perf_counter()
-    oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
-    rate = i.size / (time.perf_counter() - t0)
-    k = int(min(1 << 23, max(1 << 16, rate * target_s)))
-    i, j = sample(k)
-    t0 = time.perf_counter()
-    oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
-    dt = time.perf_counter() - t0
-    i1, j1 = sample(1 << 13)  # one core, for the per-core figure (SURVEY.md §8(d) M5)
+    n_tot, dt = 0, 0.0
+    while dt < target_s and n_tot < (1 << 23):
+        i, j = _sample_pairs(rng, ms.m, REF_CALL_PAIRS)
+        t0 = time.perf_counter()
+        oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
+        dt += time.perf_counter() - t0
+        n_tot += i.size
+    i1, j1 = _sample_pairs(rng, ms.m, 1 << 13)  # one core, for the per-core figure
     t1 = time.perf_counter()
     oracle.gcd_index_pairs(ms.N, i1, j1, nthreads=1)
     dt1 = time.perf_counter() - t1
-    return {"value": i.size / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+    # (E) on one core: calibrate, then ~4 s
+    ie, je = _sample_pairs(rng, ms.m, 1 << 11)
+    t2 = time.perf_counter()
+    oracle.approx_index_pairs(ms.N, ie, je, ms.bits, True, nthreads=1)
+    k = int(min(1 << 20, max(1 << 11, (1 << 11) / (time.perf_counter() - t2) * 4.0)))
+    ie, je = _sample_pairs(rng, ms.m, k)
+    t2 = time.perf_counter()
+    _, _, ctr = oracle.approx_index_pairs(ms.N, ie, je, ms.bits, True, nthreads=1)
+    dte = time.perf_counter() - t2
+    return {"value": n_tot / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
             "value_1core": i1.size / dt1, "us_per_gcd_1core": dt1 / i1.size * 1e6,
-            "sample": f"{i.size} seeded random (i<j) pairs of the {ms.m}-moduli workload, exact classical Euclid "
-                      f"(Knuth D), {dt:.1f}s on {cores} threads; 1-core figure on {i1.size} pairs"}
+            "sample": f"{n_tot} seeded random (i<j) pairs of the {ms.m}-moduli workload in calls of "
+                      f"{REF_CALL_PAIRS}, exact classical Euclid (Knuth D) + the O3 map, {dt:.1f}s on {cores} threads; "
+                      f"1-core figure on {i1.size} pairs",
+            "paper_algorithm_E_1core": {
+                "value": ie.size / dte, "unit": UNIT, "cores": 1, "us_per_gcd": dte / ie.size * 1e6,
+                "iterations_per_gcd": ctr[0] / ie.size, "kind": "approximate-euclid (oracle/approx_euclid.c)",
+                "paper_us_per_gcd": PAPER_E_US.get(ms.bits), "paper_hardware": "Xeon X7460, 1 thread (Table V, L491)",
+                "sample": f"{ie.size} seeded random (i<j) pairs, early-terminate, {dte:.1f}s on 1 thread"}}
 
 
 def run_reference(args):
@@ -248,14 +276,11 @@ def run_reference(args):
     import oracle
     ms = synth.config_moduli(3)
     cores = os.cpu_count() or 1
-    per_step = 1 << 18
+    per_step = REF_CALL_PAIRS
     rng = np.random.default_rng(11)
 
     def step():
-        i = rng.integers(0, ms.m, size=2 * per_step)
-        j = rng.integers(0, ms.m, size=2 * per_step)
-        keep = i < j
-        i, j = i[keep][:per_step], j[keep][:per_step]
+        i, j = _sample_pairs(rng, ms.m, per_step)
         t0 = time.perf_counter()
         G = oracle.gcd_index_pairs(ms.N, i, j, nthreads=cores)
         dt = time.perf_counter() - t0
@@ -333,7 +358,8 @@ def run_pairs(args):
     step(bg.FLAG_STATS)  # algorithmic work (untimed stats pass)
     torch.cuda.synchronize()
     ctr = dS.cpu().numpy().astype(np.int64)
-    iters, limbs = int(ctr[2]), int(ctr[4])
+    iters, limbs, slots, passw = int(ctr[2]), int(ctr[4]), int(ctr[5]), int(ctr[6])
+    eff = {"lane_efficiency": iters / slots if slots else None, "pass_word_efficiency": limbs / passw if passw else None}
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
@@ -397,7 +423,7 @@ def run_pairs(args):
                        "iterations_per_gcd": iters / m, "limb_steps_per_gcd": limbs / m,
                        "truth_ok": ok, "checked": int(m)},
             "roofline": dict(roofline(limbs, iters, m, kern_s, sms, f"pairs_kernel<{W}, exact>",
-                                      kern_total_ms / step_total_ms, None),
+                                      kern_total_ms / step_total_ms, _traffic("cfg2"), eff),
                              hbm_bytes_per_gcd_alg=3 * W * 4, hbm_GBps_alg=3 * W * 4 * m / kern_s / 1e9),
             "e2e": {"value": m_all / (float(e2e_t[0]) / args.e2e_steps), "unit": UNIT,
                     "h2d_bytes_per_step": int(A.nbytes + B.nbytes) * world, "d2h_bytes_per_step": int(A.nbytes) * world},
@@ -432,7 +458,7 @@ def cpu_baseline_pairs(A, B, target_s: float = 10.0):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -462,11 +488,18 @@ def main():
     local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    comm = None
     if world > 1:
         if BACKEND == "gloo":
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=dev)
+        comm = {"backend": dist.get_backend(), "rank": dist.get_rank(), "world": dist.get_world_size(),
+                "device": f"cuda:{local}"}
+        if BACKEND != "gloo":
+            comm["nccl_version"] = ".".join(str(x) for x in torch.cuda.nccl.version())
+        print(f"[bench] rank {comm['rank']}/{comm['world']} backend={comm['backend']} device={comm['device']}",
+              file=sys.stderr, flush=True)
     bg.bulkgcd_device_check()
 
     # ---- inputs: rank 0 generates the seeded moduli, NCCL broadcast to the others
@@ -512,11 +545,14 @@ def main():
     runner.search(bg.FLAG_STATS | algo_flag)
     torch.cuda.synchronize()
     ctr = runner.d_ctr.cpu().numpy().astype(np.int64)
-    iters, limbs = int(ctr[2]), int(ctr[4])
+    iters, limbs, slots, passw, betapos = int(ctr[2]), int(ctr[4]), int(ctr[5]), int(ctr[6]), int(ctr[7])
     if world > 1:
-        tt = torch.tensor([iters, limbs], dtype=torch.int64, device=dev)
+        tt = torch.tensor([iters, limbs, slots, passw, betapos], dtype=torch.int64, device=dev)
         _coll(dist.all_reduce, tt)
-        iters, limbs = int(tt[0]), int(tt[1])
+        iters, limbs, slots, passw, betapos = (int(x) for x in tt)
+    # SIMT efficiencies of the lockstep register kernels (the smem kernels run lanes independently)
+    eff = {"lane_efficiency": iters / slots if slots else None,
+           "pass_word_efficiency": limbs / passw if passw else None} if (W < 128 and args.algo == "E") else None
 
     k0 = torch.cuda.Event(enable_timing=True)
     k1 = torch.cuda.Event(enable_timing=True)
@@ -607,17 +643,21 @@ def main():
                        "l2": "flushed before every step (256 MiB write); inputs 2 MiB",
                        "ns_per_gcd": step_total_ms / args.steps * 1e6 / pairs,
                        "iterations_per_gcd": iters / pairs, "limb_steps_per_gcd": limbs / pairs,
+                       "beta_pos_iterations": betapos if W >= 128 else None,
+                       "ms_per_step_median": statistics.median(step_ms), "ms_per_step_min": min(step_ms),
                        "hits_ok": bool(ok), "hits": len(found), "wall_s": t_wall},
             # per-GPU kernel throughput: each rank runs 1/world of the work
             "roofline": roofline(limbs / world, iters / world, pairs / world, kern_s, sms,
                                  (f"allpairs_kernel<{W}>" if W < 128 else f"allpairs_smem_kernel<{W}>")
                                  if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
-                                 kern_total_ms / step_total_ms, _traffic()),
+                                 kern_total_ms / step_total_ms, _traffic(args.workload), eff),
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,
                     "d2h_bytes_per_step": int(d2h) * world} if e2e_value else None,
             "gpu_launches": 2 * args.steps,
             "clocks": clk.summary(),
         }
+        if comm:
+            line["config"]["comm"] = comm
         if world == 1 and not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline(ms)
         print(json.dumps(line))

@@ -12,6 +12,10 @@ two share no code; only the seeded input generators in ``synth`` serve both.
   algorithm step by step (L107, L127, L255), d-generic, with counters; used to
   pin the worked examples (Table III, the approx examples) and Table IV, and
   for per-pair iteration-count parity with the GPU.
+* :mod:`oracle.approx_euclid` (C, ``approx_euclid.c``): the same paper algorithm
+  as approx_model, d = 32, in plain C on word arrays -- the CPU (E) column of
+  Table V for bench.py's cpu_baseline; pinned per pair against
+  approx_model (tests/test_model.py).
 * :func:`rsa_hit` -- the RSA-mode result mapping.
 """
 from __future__ import annotations
@@ -26,15 +30,17 @@ from . import approx_model  # noqa: F401  (re-exported)
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "gcd_oracle.c")
+_SRC2 = os.path.join(_HERE, "approx_euclid.c")
 _SO = os.path.join(_HERE, "libgcd_oracle.so")
 _lib = None
 
 
 def build(force: bool = False) -> str:
-    """Compile the C oracle (gcc -O2) -> oracle/libgcd_oracle.so."""
-    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+    """Compile the C oracle and the C (E) baseline (gcc -O2) -> oracle/libgcd_oracle.so."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < max(os.path.getmtime(_SRC),
+                                                                       os.path.getmtime(_SRC2)):
         tmp = _SO + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-shared", "-fPIC", "-o", tmp, _SRC, "-lpthread"])
+        subprocess.check_call(["gcc", "-O2", "-shared", "-fPIC", "-o", tmp, _SRC, _SRC2, "-lpthread"])
         os.replace(tmp, _SO)
     return _SO
 
@@ -54,6 +60,10 @@ def _load():
         lib.oracle_gcd_batch.restype = ctypes.c_int
         lib.oracle_gcd_index_pairs.argtypes = [vp, vp, vp, sz, u32, vp, ctypes.c_int]
         lib.oracle_gcd_index_pairs.restype = ctypes.c_int
+        lib.oracle_approx_gcd.argtypes = [vp, vp, u32, ctypes.c_int, vp, vp]
+        lib.oracle_approx_gcd.restype = ctypes.c_long
+        lib.oracle_approx_index_pairs.argtypes = [vp, vp, vp, sz, u32, ctypes.c_int, vp, vp, vp, ctypes.c_int]
+        lib.oracle_approx_index_pairs.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -124,6 +134,34 @@ def gcd_index_pairs(N: np.ndarray, ii, jj, nthreads: int | None = None) -> np.nd
                                                   N.shape[1], G.ctypes.data, nt) != 0:
         raise RuntimeError("oracle_gcd_index_pairs failed")
     return G
+
+
+def approx_gcd(a: int, b: int, bits: int, early: bool) -> tuple[int, int]:
+    """(result, iterations) of the C Approximate Euclid (approx_euclid.c) on one pair of
+    `bits`-bit operands: early=True is RSA mode on odd inputs (g or 1), early=False the
+    exact gcd of any inputs (L41)."""
+    n = bits // 32
+    A, B, G = _limbs(a, n), _limbs(b, n), np.zeros(n, np.uint32)
+    it = _load().oracle_approx_gcd(A.ctypes.data, B.ctypes.data, n, bits if early else 0, G.ctypes.data, None)
+    if it < 0:
+        raise ValueError("operand too large")
+    return _int(G), int(it)
+
+
+def approx_index_pairs(N: np.ndarray, ii, jj, bits: int, early: bool = True, nthreads: int = 1):
+    """The C (E) baseline over index pairs: (G uint32[k, W], iterations uint32[k],
+    [sum iterations, sum limb-steps, beta>0 iterations])."""
+    N = np.ascontiguousarray(N, dtype=np.uint32)
+    ii = np.ascontiguousarray(ii, dtype=np.uint64)
+    jj = np.ascontiguousarray(jj, dtype=np.uint64)
+    G = np.zeros((ii.size, N.shape[1]), np.uint32)
+    it = np.zeros(ii.size, np.uint32)
+    ctr = np.zeros(3, np.uint64)
+    if ii.size and _load().oracle_approx_index_pairs(N.ctypes.data, ii.ctypes.data, jj.ctypes.data, ii.size,
+                                                     N.shape[1], bits if early else 0, G.ctypes.data, it.ctypes.data,
+                                                     ctr.ctypes.data, nthreads) != 0:
+        raise RuntimeError("oracle_approx_index_pairs failed")
+    return G, it, [int(x) for x in ctr]
 
 
 def bitlen_rows(G: np.ndarray) -> np.ndarray:

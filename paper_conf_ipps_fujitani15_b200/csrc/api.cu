@@ -215,7 +215,7 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
                     uint64_t cap, unsigned long long *counters, unsigned flags, cudaStream_t st) {
     CK(cudaMemsetAsync(counters, 0, 8 * sizeof(unsigned long long), st));
     if (c1 <= c0) return 0;
-    AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16, nullptr};
+    AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
     if constexpr (W >= 128) {
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     } else {
@@ -225,12 +225,8 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if ((flags & BULKGCD_FLAG_SMEM) || (flags & BULKGCD_FLAG_ALGO_MASK))
         return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
     uint64_t warps = c1 - c0;
-    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * Occ<W>::blocks, (warps + WARPS_PER_CTA - 1) / WARPS_PER_CTA);
-    DBuf park;  // freed stream-ordered after the kernel
-    if constexpr (ParkCfg<W>::gmem) {
-        CK(park.alloc(grid * WARPS_PER_CTA * sizeof(ParkPool<W>), st));
-        a.park = park.p;
-    }
+    constexpr int wpc = ApCfg<W>::warps_per_cta;
+    uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * ApCfg<W>::blocks, (warps + wpc - 1) / wpc);
     constexpr size_t smem = allpairs_smem_bytes<W>();
     static PerDeviceOnce attr_once;  // dynamic shared memory opt-in, per device
     if (int rc = attr_once.run([]() -> int {
@@ -239,8 +235,8 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
             return 0;
         }))
         return rc;
-    if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, THREADS, smem, st>>>(a);
-    else allpairs_kernel<W, false><<<(unsigned)grid, THREADS, smem, st>>>(a);
+    if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, ApCfg<W>::threads, smem, st>>>(a);
+    else allpairs_kernel<W, false><<<(unsigned)grid, ApCfg<W>::threads, smem, st>>>(a);
     CK(cudaGetLastError());
     return 0;
     }

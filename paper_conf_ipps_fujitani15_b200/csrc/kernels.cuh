@@ -166,12 +166,11 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // pass (B + alpha*A~ + alpha).  The roles alternate strictly, which keeps A complemented;
 // the rare cold-section code that reads the operand registers (fix-ups, the hit sink)
 // sees plain values (A is complemented around it).
-template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, class Parker, bool CMPL = false>
+template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, bool CMPL = false>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
-                                            uint64_t &tB, bool live, Cond cond, Sink &sink, Parker &pk, int s0,
+                                            uint64_t &tB, bool live, Cond cond, Sink &sink, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
                                             uint32_t &passw) {
-    static_assert(!(CMPL && Parker::enabled), "complement form: no straggler parking");
     using CmA = std::integral_constant<int, CMPL ? 1 : 0>;  // hot_iter pass form with A updated
     using CmB = std::integral_constant<int, CMPL ? 2 : 0>;  // ... with B updated
     int s = s0;
@@ -202,11 +201,6 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         live = run;
         unsigned brun = __ballot_sync(FULL, run);
         if (brun == 0u) return false;
-        if (Parker::enabled && pk.wants(__popc(brun))) {  // few stragglers left: park them, free the warp
-            pk.park(run, brun, X, Y, lX, tX, lY, tY, s, sink);
-            live = false;
-            return false;
-        }
         int L = __reduce_max_sync(FULL, (unsigned)(run ? lX : 0));
         while (W - s > L) {
             shift_up_1<W>(A);
@@ -242,9 +236,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         }
         if (!any_top) {  // the warp length dropped (lanes finished or shrank): realign one word in place
             unsigned brun = __ballot_sync(FULL, run);
-            // go cold if nobody runs, or to park the last few stragglers (checked only here:
-            // the warp length drops when the longest lanes finish)
-            if ((brun == 0u) | (Parker::enabled && pk.wants(__popc(brun)))) {
+            if (brun == 0u) {  // nobody runs: go cold (the cohort ends there)
                 fix = fix_code(live, full, post, lt);
                 return true;
             }
@@ -286,61 +278,6 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         }
     }
 }
-
-// ---- straggler parking (SIMT lane efficiency; SURVEY.md §7 H-d)
-// A lockstep cohort runs as long as its slowest lane: ~10% of lane-slots are
-// idle.  When at most K lanes are still running, the warp parks them in a
-// per-warp shared-memory pool (state: both operands, lengths, tops, i, j) and
-// takes new work; 32 parked lanes later run together as one cohort.
-struct NoPark {
-    static constexpr bool enabled = false;
-    __device__ __forceinline__ bool wants(unsigned) const { return false; }
-    template <int W, class Sink>
-    __device__ __forceinline__ void park(bool, unsigned, uint32_t (&)[W], uint32_t (&)[W], int, uint64_t, int,
-                                         uint64_t, int, Sink &) {}
-};
-
-template <int W>
-struct ParkPool {  // per warp, in shared memory; word-interleaved by slot (conflict-free)
-    uint32_t x[W * 32];
-    uint32_t y[W * 32];
-    uint32_t meta[8 * 32];  // lX, lY, tX.lo, tX.hi, tY.lo, tY.hi, i, j
-};
-
-template <int W>
-struct Parker {
-    static constexpr bool enabled = true;
-    ParkPool<W> *pool;
-    unsigned npool;  // warp-uniform
-    unsigned K;      // park when <= K lanes still run (0: never)
-    __device__ __forceinline__ bool wants(unsigned nrun) const { return nrun <= K && npool + nrun <= 32u; }
-    template <class Sink>
-    __device__ __forceinline__ void park(bool run, unsigned brun, uint32_t (&X)[W], uint32_t (&Y)[W], int lX,
-                                         uint64_t tX, int lY, uint64_t tY, int s, Sink &sink) {
-        const unsigned lane = threadIdx.x & 31;
-        unsigned slot = npool + __popc(brun & ((1u << lane) - 1u));
-        if (run) {
-#pragma unroll
-            for (int k = 0; k < W; ++k) {
-                if (k >= s) {
-                    pool->x[(k - s) * 32 + slot] = X[k];  // least significant word first
-                    pool->y[(k - s) * 32 + slot] = Y[k];
-                }
-            }
-            uint32_t *m = pool->meta + slot;
-            m[0] = (uint32_t)lX;
-            m[32] = (uint32_t)lY;
-            m[64] = lo32(tX);
-            m[96] = hi32(tX);
-            m[128] = lo32(tY);
-            m[160] = hi32(tY);
-            m[192] = sink.i;
-            m[224] = sink.j;
-        }
-        npool += __popc(brun);
-        __syncwarp();
-    }
-};
 
 // RSA-mode loop condition (early-terminate, L243/L251/L255): continue while Y
 // has at least s/2 bits.
@@ -496,9 +433,8 @@ __global__ void BULKGCD_BOUNDS(W, true) pairs_kernel(PairsArgs a) {
             bool live = valid;
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkRsa<W> sink{a.G, i, a.m_pad};
-            NoPark np;
-            euclid_loop<W, STATS, false, true>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow, limbs,
-                                         slots, passw);
+            euclid_loop<W, STATS, false, true>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, 0, iters, nslow, limbs,
+                                               slots, passw);
         } else {
             int k2 = 0;
             bool known = false;
@@ -514,9 +450,8 @@ __global__ void BULKGCD_BOUNDS(W, true) pairs_kernel(PairsArgs a) {
             }
             setup_pair<W>(A, B, lA, tA, lB, tB);
             PairsSinkExact<W> sink{a.G, i, a.m_pad, k2, false, 0, 0};
-            NoPark np;
-            euclid_loop<W, STATS, true, false>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, np, 0, iters, nslow, limbs, slots,
-                                        passw);
+            euclid_loop<W, STATS, true, false>(A, B, lA, tA, lB, tB, live, ExactCond{}, sink, 0, iters, nslow, limbs, slots,
+                                               passw);
             // 64-bit tail: Case 1 of approx (lX <= 2): alpha = X div Y, exactly (L127).
             if (sink.tail) {
                 uint64_t x = sink.x64, y = sink.y64;
@@ -574,7 +509,6 @@ struct AllPairsArgs {
     unsigned long long *hit_count;
     unsigned long long *stats;     // optional [sum iterations, slow steps, limb-steps]
     int half;
-    void *park;                    // straggler pools in global memory (ParkCfg<W>::gmem), one per warp
 };
 
 template <int W>
@@ -622,25 +556,25 @@ struct StageBuf {
     uint32_t col[W];
 };
 
-#ifndef BULKGCD_PARK_K
-#define BULKGCD_PARK_K 0  // straggler parking: measured a wash on B200, off by default
+// CTA shape of the all-pairs kernel, by width: warps are independent (each claims its
+// own cohorts from the atomic cursor), so the CTA size only decides how the resident
+// warps are grouped.  W <= 32: one warp per CTA, 20 CTAs/SM (cfg3 246.7 -> 240.9 ms against
+// 4-warp CTAs at the same 20 warps/SM, 96 registers; 19: 242.5, 21 (80 registers): 244.6).
+// W = 64: 4-warp CTAs (one-warp CTAs: cfg4 851 -> 1,592 ms).
+#ifndef BULKGCD_AP_THREADS_NARROW
+#define BULKGCD_AP_THREADS_NARROW 32
 #endif
-#ifndef BULKGCD_PARK_GMEM
-#define BULKGCD_PARK_GMEM 1  // pool in global memory (per warp, L2-resident), not next to the TMA buffers
-#endif
-// Parking pool: in shared memory only where it fits next to the TMA buffers at the
-// kernel's occupancy; in global memory (AllPairsArgs::park, one pool per warp) otherwise.
 template <int W>
-struct ParkCfg {
-    static constexpr bool on = (BULKGCD_PARK_GMEM ? W <= 64 : W <= 32) && (BULKGCD_PARK_K > 0);
-    static constexpr bool gmem = on && BULKGCD_PARK_GMEM;
-    static constexpr size_t pool_bytes = (on && !gmem) ? sizeof(ParkPool<W>) : 0;
+struct ApCfg {
+    static constexpr int threads = W <= 32 ? BULKGCD_AP_THREADS_NARROW : 128;
+    static constexpr int warps_per_cta = threads / 32;
+    static constexpr int warps = Occ<W>::warps;  // resident warps per SM (register budget)
+    static constexpr int blocks = warps / warps_per_cta > 0 ? warps / warps_per_cta : 1;
 };
 
 template <int W>
 constexpr size_t allpairs_smem_bytes() {
-    return (THREADS / 32) * (2 * sizeof(StageBuf<W>) + ParkCfg<W>::pool_bytes) +
-           (THREADS / 32) * 2 * sizeof(unsigned long long);
+    return ApCfg<W>::warps_per_cta * (2 * sizeof(StageBuf<W>) + 2 * sizeof(unsigned long long));
 }
 
 __device__ __forceinline__ uint32_t smem_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -692,17 +626,19 @@ __device__ __forceinline__ void cohort_coords(uint64_t c, uint64_t n, uint64_t &
 template <int W>
 __host__ __device__ constexpr bool allpairs_cmpl() { return W >= BULKGCD_ALLPAIRS_CMPL_MIN_W; }
 
+#ifdef BULKGCD_MAXNREG
+#define BULKGCD_AP_BOUNDS(W) __maxnreg__(BULKGCD_MAXNREG)
+#else
+#define BULKGCD_AP_BOUNDS(W) __launch_bounds__(ApCfg<W>::threads, ApCfg<W>::blocks)
+#endif
+
 template <int W, bool STATS>
-__global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
+__global__ void BULKGCD_AP_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     StageBuf<W> *buf = reinterpret_cast<StageBuf<W> *>(smem_raw) + 2 * warp;
-    unsigned char *after_bufs = smem_raw + (THREADS / 32) * 2 * sizeof(StageBuf<W>);
-    ParkPool<W> *pool = ParkCfg<W>::gmem  // valid only if ParkCfg<W>::on
-                            ? reinterpret_cast<ParkPool<W> *>(a.park) + (blockIdx.x * (THREADS / 32) + warp)
-                            : reinterpret_cast<ParkPool<W> *>(after_bufs) + warp;
     unsigned long long *bar =
-        reinterpret_cast<unsigned long long *>(after_bufs + (THREADS / 32) * ParkCfg<W>::pool_bytes) + 2 * warp;
+        reinterpret_cast<unsigned long long *>(smem_raw + ApCfg<W>::warps_per_cta * 2 * sizeof(StageBuf<W>)) + 2 * warp;
     if (lane == 0) {
         mbar_init(&bar[0], 1);
         mbar_init(&bar[1], 1);
@@ -728,50 +664,10 @@ __global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
         return true;
     };
 
-    Parker<W> pk{pool, 0u, ParkCfg<W>::on ? (unsigned)BULKGCD_PARK_K : 0u};
-
-    // Run up to 32 parked stragglers as one cohort (top slots of the pool).
-    auto run_parked = [&](bool allow_park) {
-        unsigned take = pk.npool < 32u ? pk.npool : 32u;
-        unsigned slot = pk.npool - take + lane;
-        bool live = (unsigned)lane < take;
-        const uint32_t *m = pool->meta + slot;
-        int lA = live ? (int)m[0] : 0, lB = live ? (int)m[32] : 0;
-        uint64_t tA = live ? ((uint64_t)m[96] << 32 | m[64]) : 0, tB = live ? ((uint64_t)m[160] << 32 | m[128]) : 0;
-        uint32_t pi = live ? m[192] : 0u, pj = live ? m[224] : 0u;
-        int L = (int)__reduce_max_sync(FULL, (unsigned)lA);
-        int s = W - L;
-        uint32_t A[W], B[W];
-#pragma unroll
-        for (int k = 0; k < W; ++k) {  // pool words beyond a lane's own lengths are stale: read as zero
-            A[k] = (live & (k >= s) & (k - s < lA)) ? pool->x[(k - s) * 32 + slot] : 0u;
-            B[k] = (live & (k >= s) & (k - s < lB)) ? pool->y[(k - s) * 32 + slot] : 0u;
-        }
-        __syncwarp();
-        pk.npool -= take;
-        unsigned K = pk.K;
-        if (!allow_park) pk.K = 0;
-        HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, pi, pj};
-        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, s, iters, nslow, limbs,
-                                     slots, passw);
-        pk.K = K;
-    };
-
     int slot = 0;
     uint64_t c, b, j;
     bool have = claim(0, c, b, j);
-    for (;;) {
-        if (ParkCfg<W>::on && pk.npool >= 32u) {
-            run_parked(true);
-            continue;
-        }
-        if (!have) {
-            if (ParkCfg<W>::on && pk.npool > 0u) {  // drain: no more fresh work
-                run_parked(false);
-                continue;
-            }
-            break;
-        }
+    while (have) {
         uint64_t c2, b2, j2;
         bool have2 = claim(slot ^ 1, c2, b2, j2);  // prefetch the next cohort
         mbar_wait(&bar[slot], phase[slot]);
@@ -789,14 +685,8 @@ __global__ void BULKGCD_BOUNDS(W, false) allpairs_kernel(AllPairsArgs a) {
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
-        if (ParkCfg<W>::on) {
-            euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, decltype(pk)>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, pk, 0, iters, nslow,
-                                         limbs, slots, passw);
-        } else {
-            NoPark np;
-            euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, NoPark, allpairs_cmpl<W>()>(
-                A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, np, 0, iters, nslow, limbs, slots, passw);
-        }
+        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, allpairs_cmpl<W>()>(
+            A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, 0, iters, nslow, limbs, slots, passw);
         slot ^= 1;
         have = have2;
         c = c2;

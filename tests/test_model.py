@@ -167,3 +167,35 @@ def test_table4_binary_columns(bits, npairs):
             assert abs(arr.mean() - paper) <= 3 * se + 0.05, (col, mode, bits, arr.mean(), paper, se)
     g = [am.binary_euclid(N[k], N[k + 1]).gcd for k in range(50)]
     assert g == [math.gcd(N[k], N[k + 1]) for k in range(50)]
+
+
+@pytest.mark.parametrize("bits", [512, 1024, 2048, 4096])
+def test_c_approx_euclid_matches_model(bits):
+    """oracle/approx_euclid.c (the CPU (E) column of Table V) is the
+    paper's algorithm: per pair, the same result and the same iteration count as the
+    model, in RSA mode on synthetic moduli and in exact mode on the rare-path operands
+    (Cases 1-3, beta > 0, rshift >= 32, even and zero inputs)."""
+    ms = synth.moduli(24, bits, seed=900 + bits, n_planted_pairs=2)
+    N = synth.ints(ms.N)
+    for i in range(len(N)):
+        for j in range(i + 1, min(len(N), i + 6)):
+            t = am.gcd_rsa(N[i], N[j], bits)
+            assert oracle.approx_gcd(N[i], N[j], bits, True) == (t.gcd, t.iterations), (bits, i, j)
+    A, B = synth.mixed_pairs(220, bits, seed=77 + bits)
+    for a, b in zip(A, B):
+        t = am.gcd_exact(a, b)
+        assert oracle.approx_gcd(a, b, bits, False) == (t.gcd, t.iterations), (bits, a, b)
+        assert t.gcd == math.gcd(a, b)
+
+
+def test_c_approx_euclid_batch_and_counters(cfg1):
+    """The batch entry (threads) equals the single-pair calls; its counters equal the
+    model's iterations, limb-steps and beta > 0 counts (M2's units)."""
+    ii, jj = np.triu_indices(cfg1.m, k=1)
+    G, it, ctr = oracle.approx_index_pairs(cfg1.N, ii, jj, 1024, True, nthreads=4)
+    N = synth.ints(cfg1.N)
+    tr = [am.gcd_rsa(N[i], N[j], 1024) for i, j in zip(ii, jj)]
+    assert [int(x) for x in it] == [t.iterations for t in tr]
+    assert ctr == [sum(t.iterations for t in tr), sum(t.limb_steps for t in tr), sum(t.beta_pos for t in tr)]
+    hits = sorted((int(i), int(j), synth.to_int(G[k])) for k, (i, j) in enumerate(zip(ii, jj)) if synth.to_int(G[k]) != 1)
+    assert hits == cfg1.truth
