@@ -28,6 +28,62 @@ def band(total: int, world: int, rank: int) -> tuple[int, int]:
     return total * rank // world, total * (rank + 1) // world
 
 
+def _pairs_in_first(o):
+    """Pairs in the first o cohorts of a row block: cohort d (1-based) holds min(32, d) pairs
+    (lanes 32b + t < j with j = 32b + d), so sum_{d <= o} min(32, d)."""
+    o = np.asarray(o, dtype=np.int64)
+    return np.where(o <= 32, o * (o + 1) // 2, 528 + 32 * (o - 32))
+
+
+def _row_block_prefix(n: int):
+    """(cohort prefix P[b], pair prefix Q[b]) over row blocks b = 0..nb (cohorts of row block b
+    are j = 32b+1 .. n-1, ordered as in include/bulkgcd.h's cohort ids)."""
+    nb = (n + 31) // 32
+    b = np.arange(nb, dtype=np.int64)
+    cnt = np.maximum(n - 1 - 32 * b, 0)
+    P = np.concatenate([[0], np.cumsum(cnt)])
+    Q = np.concatenate([[0], np.cumsum(_pairs_in_first(cnt))])
+    return P, Q
+
+
+def pairs_before(c: int, n: int) -> int:
+    """Number of pairs i < j in the cohorts [0, c) of an n-moduli all-pairs search."""
+    P, Q = _row_block_prefix(n)
+    c = min(max(int(c), 0), int(P[-1]))
+    b = int(np.searchsorted(P, c, side="right")) - 1
+    b = min(b, len(P) - 2) if len(P) > 1 else 0
+    return int(Q[b] + _pairs_in_first(c - P[b])) if len(P) > 1 else 0
+
+
+def band_pairs(n: int, world: int, rank: int) -> tuple[int, int]:
+    """Row band of `rank` balanced by PAIRS (= work): the cohort range
+    [c_r, c_{r+1}) with c_r the first cohort at which the pair count reaches
+    r * n(n-1)/2 / world.  Bands tile [0, cohort_total) and each holds its share of the
+    pairs to within one cohort (< 32 pairs), whereas equal cohort counts (band()) give
+    up to ~0.1% more pairs to the first bands (their rows have fewer partial cohorts)."""
+    if world < 1 or not 0 <= rank < world:
+        raise ValueError("bad world/rank")
+    P, Q = _row_block_prefix(n)
+    total_pairs = n * (n - 1) // 2
+
+    def cut(r):
+        if r == 0:
+            return 0
+        if r == world:
+            return int(P[-1])
+        t = -(-r * total_pairs // world)  # ceil(r * total / world)
+        b = int(np.searchsorted(Q, t, side="left")) - 1  # Q[b] < t <= Q[b+1]
+        need = t - int(Q[b])
+        o = int(np.ceil((np.sqrt(8 * need + 1) - 1) / 2)) if need <= 528 else 32 + -(-(need - 528) // 32)
+        while o > 0 and _pairs_in_first(o - 1) >= need:
+            o -= 1
+        while _pairs_in_first(o) < need:
+            o += 1
+        return int(P[b]) + o
+
+    return cut(rank), cut(rank + 1)
+
+
 class AllPairsBand:
     """Device-resident state for one GPU's band of the all-pairs search."""
 
@@ -42,7 +98,7 @@ class AllPairsBand:
         self.d_N = torch.empty(self.h_N.shape, dtype=torch.int32, device=self.device)
         self.d_blk = torch.empty(bulkgcd_blocked_words(self.n, bits), dtype=torch.int32, device=self.device)
         self.total = bulkgcd_cohort_count(self.n)
-        self.c0, self.c1 = band(self.total, world, rank)
+        self.c0, self.c1 = band_pairs(self.n, world, rank)
         self.cap = hit_cap
         self.d_hits = torch.empty(self.cap * (2 + self.W), dtype=torch.int32, device=self.device)
         self.d_ctr = torch.zeros(8, dtype=torch.int64, device=self.device)

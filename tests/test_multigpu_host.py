@@ -10,7 +10,7 @@ import torch
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
-from paper_conf_ipps_fujitani15_b200.dist import band, gather_hits, records_to_hits
+from paper_conf_ipps_fujitani15_b200.dist import band, band_pairs, gather_hits, pairs_before, records_to_hits
 
 
 def test_band_covers_exactly_once_and_balances():
@@ -24,6 +24,43 @@ def test_band_covers_exactly_once_and_balances():
             assert max(sizes) - min(sizes) <= 1
     with pytest.raises(ValueError):
         band(10, 2, 2)
+
+
+def _cohort_pairs_brute(n):
+    """Pairs per cohort id by direct enumeration of include/bulkgcd.h's cohort order."""
+    out = []
+    for b in range((n + 31) // 32):
+        for j in range(32 * b + 1, n):
+            out.append(sum(1 for t in range(32) if 32 * b + t < j))
+    return np.array(out, dtype=np.int64)
+
+
+def test_pairs_before_matches_enumeration():
+    for n in (2, 3, 31, 32, 33, 64, 65, 100, 257):
+        cp = _cohort_pairs_brute(n)
+        assert cp.sum() == n * (n - 1) // 2
+        pre = np.concatenate([[0], np.cumsum(cp)])
+        for c in range(len(cp) + 1):
+            assert pairs_before(c, n) == pre[c], (n, c)
+
+
+@pytest.mark.parametrize("n", [64, 257, 16384, 65536])
+def test_band_pairs_balance(n):
+    """SURVEY.md §8(e) G1 at the configs' sizes (cfg3: 16,384 moduli; cfg5: 65,536 for the
+    8-GPU run): the bands of N = 2/4/8 ranks tile the cohort range and each holds its
+    share of the n(n-1)/2 pairs to within one cohort (< 32 pairs)."""
+    from paper_conf_ipps_fujitani15_b200 import bulkgcd_cohort_count  # host helper of the C ABI
+    total_c = (n + 31) // 32 * (n - 1) - 16 * ((n + 31) // 32) * ((n + 31) // 32 - 1)
+    total_p = n * (n - 1) // 2
+    assert bulkgcd_cohort_count(n) == total_c  # the C ABI's host helper (no GPU needed)
+    for world in (1, 2, 3, 4, 8):
+        cuts = [band_pairs(n, world, r) for r in range(world)]
+        assert cuts[0][0] == 0 and cuts[-1][1] == total_c
+        for (a0, a1), (b0, b1) in zip(cuts, cuts[1:]):
+            assert a1 == b0 and a0 <= a1
+        for r, (c0, c1) in enumerate(cuts):
+            got = pairs_before(c1, n) - pairs_before(c0, n)
+            assert abs(got - total_p / world) < 32 + 1e-9, (n, world, r, got, total_p / world)
 
 
 def _free_port():
