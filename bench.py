@@ -59,6 +59,9 @@ WORKLOADS = {
             "(the paper's 512-bit Table V workload; SURVEY.md §8(f) N1, not a BASELINE.json config)",
     "cfg7": "cfg7: all-pairs 4096-bit RSA moduli, n=512 (130,816 pairs), 4 planted shared primes "
             "(shared-memory kernels; SURVEY.md §8(f) N1, not a BASELINE.json config)",
+    "cfg8": "cfg8: all-pairs 4096-bit moduli, n=16384 (134,209,536 pairs: the paper's Table V 4096-bit size, "
+            "PAPER.md L451/L493), 8 planted shared factors; n = p*q from random odd 2048-bit cofactors "
+            "(SURVEY.md §8(f) N1, not a BASELINE.json config)",
     "cfg2": "cfg2: 2^20 independent 1024-bit pair GCDs, exact mode (bulkgcd_pairs; the first 2^20 pairs i<j "
             "of a 1,449-moduli pool with 2 planted shared primes; BASELINE.json configs[1])",
 }
@@ -504,7 +507,8 @@ def main():
 
     # ---- inputs: rank 0 generates the seeded moduli, NCCL broadcast to the others
     k = int(args.workload[3:])
-    bits = synth.CONFIGS[k]["bits"]
+    cfgk = synth.CONFIG8 if k == 8 else synth.CONFIGS[k]
+    bits = cfgk["bits"]
     W = bits // 32
     metric = f"{bits}-bit GCDs/sec (all-pairs)"
     if rank == 0:
@@ -512,7 +516,7 @@ def main():
         N = ms.N
         truth = ms.truth
     else:
-        N = np.zeros((synth.CONFIGS[k]["m"], W), np.uint32)
+        N = np.zeros((cfgk["m"], W), np.uint32)
         truth = None
     if world > 1:
         t = torch.from_numpy(N.view(np.int32)).to(dev)
@@ -591,7 +595,14 @@ def main():
     else:
         allrec = local_hits
     found = bgd.records_to_hits(allrec.cpu().numpy(), bits).as_list()
-    ok = (found == truth) if rank == 0 else True
+    if rank != 0:
+        ok = True
+    elif k == 8:  # cofactor moduli: the planted pairs, each g a >= bits/2-bit common divisor (exact division)
+        Ni = [synth.to_int(r) for r in N]
+        ok = [(i, j) for i, j, _ in found] == [(a, b) for a, b, _ in truth] and all(
+            g.bit_length() >= bits // 2 and Ni[i] % g == 0 and Ni[j] % g == 0 for i, j, g in found)
+    else:
+        ok = found == truth
 
     tot_ms = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
     if world > 1:

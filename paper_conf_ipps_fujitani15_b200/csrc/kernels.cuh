@@ -709,7 +709,9 @@ template <int W, bool RSA, bool STATS, int ALG>
 __global__ void __launch_bounds__(SM_THREADS) pairs_smem_kernel(PairsArgs a) {
     extern __shared__ __align__(16) uint32_t sbuf[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t *wb = sbuf + (size_t)warp * 2 * W * 32;
+    constexpr int SW = smem_stride_words<W>();
+    uint32_t *wb = sbuf + (size_t)warp * 2 * SW * 32;
+    for (int k = W; k < SW; ++k) wb[k * 32 + lane] = wb[(SW + k) * 32 + lane] = 0u;  // zero pad (s_update_ls)
     uint32_t iters = 0, rare = 0, limbs = 0, betapos = 0;
     for (;;) {
         unsigned long long c = 0;
@@ -718,13 +720,46 @@ __global__ void __launch_bounds__(SM_THREADS) pairs_smem_kernel(PairsArgs a) {
         if (c * 32 >= a.m) break;
         uint64_t i = c * 32 + lane;
         bool valid = i < a.m;
-        SOp X{wb + lane}, Y{wb + W * 32 + lane};
+        SOp X{wb + lane}, Y{wb + SW * 32 + lane};
         for (int k = 0; k < W; ++k) {
             X[k] = valid ? a.A[(uint64_t)k * a.m_pad + i] : 0u;
             Y[k] = valid ? a.B[(uint64_t)k * a.m_pad + i] : 0u;
         }
         uint32_t it0 = iters;
-        if (valid) {
+        if (ALG == ALG_APPROX) {  // lockstep loop: every lane of the warp takes part
+            int lX = 0, lY = 0, k2 = 0;
+            uint64_t tX = 0, tY = 0;
+            bool go = valid;
+            if (!RSA && valid) {
+                int la = s_len(X, W), lb = s_len(Y, W);
+                if (la == 0 || lb == 0) {  // gcd(x, 0) = x
+                    SOp Z = la ? X : Y;
+                    s_write_shifted(a.G + i, a.m_pad, Z, la ? la : lb, 0, W);
+                    go = false;
+                } else {  // L41: strip the common power of two k2 and every other factor 2
+                    int ca = s_ctz(X, la), cb = s_ctz(Y, lb);
+                    k2 = ca < cb ? ca : cb;
+                    s_rshift(X, la);
+                    s_rshift(Y, lb);
+                }
+            }
+            if (go) s_setup(X, Y, lX, tX, lY, tY, W);
+            s_euclid_ls<!RSA, STATS>(X, Y, lX, tX, lY, tY, a.half, go, iters, rare, limbs, betapos);
+            if (go) {
+                if (RSA) {
+                    if (lY == 0) s_write_shifted(a.G + i, a.m_pad, X, lX, 0, W);  // g = X (L251)
+                    else for (int w = 0; w < W; ++w) a.G[i + (uint64_t)w * a.m_pad] = w == 0 ? 1u : 0u;
+                } else {
+                    if (lY != 0) {  // Case 1 tail (lX <= 2)
+                        uint64_t g = s_tail64<STATS>(s_value64(X, lX), s_value64(Y, lY), iters, limbs);
+                        X[0] = (uint32_t)g;
+                        X[1] = (uint32_t)(g >> 32);
+                        lX = g >> 32 ? 2 : (g ? 1 : 0);
+                    }
+                    s_write_shifted(a.G + i, a.m_pad, X, lX, k2, W);
+                }
+            }
+        } else if (valid) {
             int lX, lY;
             uint64_t tX, tY;
             if (RSA) {
@@ -771,7 +806,9 @@ template <int W, bool STATS, int ALG>
 __global__ void __launch_bounds__(SM_THREADS) allpairs_smem_kernel(AllPairsArgs a) {
     extern __shared__ __align__(16) uint32_t sbuf[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t *wb = sbuf + (size_t)warp * 2 * W * 32;
+    constexpr int SW = smem_stride_words<W>();
+    uint32_t *wb = sbuf + (size_t)warp * 2 * SW * 32;
+    for (int k = W; k < SW; ++k) wb[k * 32 + lane] = wb[(SW + k) * 32 + lane] = 0u;  // zero pad (s_update_ls)
     uint32_t iters = 0, rare = 0, limbs = 0, betapos = 0;
     for (;;) {
         unsigned long long cc = 0;
@@ -782,14 +819,17 @@ __global__ void __launch_bounds__(SM_THREADS) allpairs_smem_kernel(AllPairsArgs 
         cohort_coords(c, a.n, b, j);
         uint64_t i = 32 * b + lane;
         bool live = i < j;
-        SOp X{wb + lane}, Y{wb + W * 32 + lane};
+        SOp X{wb + lane}, Y{wb + SW * 32 + lane};
         for (int k = 0; k < W; ++k) {
             X[k] = a.N_blk[(b * W + k) * 32 + lane];  // one coalesced 128-byte row per word
             Y[k] = a.N_rm[j * W + k];                 // the column modulus (broadcast)
         }
         int lX = 0, lY = 0;
         uint64_t tX = 0, tY = 0;
-        if (live) {
+        if (ALG == ALG_APPROX) {  // lockstep loop: every lane of the warp takes part
+            if (live) s_setup(X, Y, lX, tX, lY, tY, W);
+            s_euclid_ls<false, STATS>(X, Y, lX, tX, lY, tY, a.half, live, iters, rare, limbs, betapos);
+        } else if (live) {
             s_setup(X, Y, lX, tX, lY, tY, W);
             s_euclid<false, STATS, ALG>(X, Y, lX, tX, lY, tY, a.half, iters, rare, limbs, betapos);
         }

@@ -26,6 +26,8 @@
 #pragma once
 #include <cstdint>
 
+#include "euclid.cuh"  // div_floor_est / div_floor_fix
+
 namespace bulkgcd {
 
 // Algorithms (the paper's comparison columns, same harness):
@@ -34,11 +36,17 @@ namespace bulkgcd {
 //   ALG_BINARY       (C) Binary Euclid, L57: X <- X/2 | Y <- Y/2 | X <- (X - Y)/2
 enum { ALG_APPROX = 0, ALG_FAST_BINARY = 1, ALG_BINARY = 2 };
 
-constexpr int SM_THREADS = 64;  // 2 warps per CTA: 2 x 2 x W x 32 x 4 bytes = 64 KiB of operands at W = 128
+constexpr int SM_THREADS = 64;  // 2 warps per CTA: 2 x 2 x (W + SM_PAD) x 32 x 4 bytes = 68 KiB at W = 128
+// Zero words above each operand buffer: the lockstep pass (s_update_ls) runs in 4-limb chunks up to
+// 3 words past the longest operand and prefetches the next chunk (up to 8 past), all reading zeros.
+constexpr int SM_PAD = 8;
+
+template <int W>
+__host__ __device__ constexpr int smem_stride_words() { return W + SM_PAD; }  // words per operand buffer
 
 template <int W>
 constexpr size_t smem_operand_bytes() {
-    return (size_t)(SM_THREADS / 32) * 2 * W * 32 * sizeof(uint32_t);
+    return (size_t)(SM_THREADS / 32) * 2 * smem_stride_words<W>() * 32 * sizeof(uint32_t);
 }
 
 template <int W>
@@ -91,20 +99,31 @@ __device__ __forceinline__ void s_rshift(SOp x, int n) {
     }
 }
 
-// approx(X, Y) of L127 for lX >= 3 (Cases 2-4; Case 1 is the 64-bit tail).
+// approx(X, Y) of L127 for lX >= 3 (Cases 2-4; Case 1 is the 64-bit tail).  Every case is
+// one quotient num div den < 2^32 (L133); it is taken exactly as in the register kernels: an
+// FP64 estimate (div_floor_est) and, for the rare estimates within 2^-16 of an integer, the
+// exact 96-bit check (div_floor_fix) -- instead of a 64-bit integer division subroutine.
 __device__ __forceinline__ void s_approx(int lX, uint64_t tX, int lY, uint64_t tY, uint32_t &alpha, int &beta) {
     uint32_t x1 = (uint32_t)(tX >> 32), y1 = (uint32_t)(tY >> 32);
-    uint64_t a;
+    uint64_t num = tX, den;
     if (lY == 1) {
-        if (x1 >= y1) { a = x1 / y1; beta = lX - 1; }                         // Case 2-A
-        else { a = tX / y1; beta = lX - 2; }                                  // Case 2-B
+        if (x1 >= y1) { num = x1; den = y1; beta = lX - 1; }                  // Case 2-A
+        else { den = y1; beta = lX - 2; }                                     // Case 2-B
     } else if (lY == 2) {
-        if (tX >= tY) { a = tX / tY; beta = lX - 2; }                         // Case 3-A
-        else { a = tX / ((uint64_t)y1 + 1); beta = lX - 3; }                  // Case 3-B
-    } else if (tX > tY) { a = tX / (tY + 1); beta = lX - lY; }              // Case 4-A
-    else if (lX > lY) { a = tX / ((uint64_t)y1 + 1); beta = lX - lY - 1; }  // Case 4-B
-    else { a = 1; beta = 0; }                                                 // Case 4-C
-    alpha = (uint32_t)a;  // < 2^32 outside Case 1 (L133); the bound alpha*D^beta <= X div Y is L123's
+        if (tX >= tY) { den = tY; beta = lX - 2; }                            // Case 3-A
+        else { den = (uint64_t)y1 + 1; beta = lX - 3; }                       // Case 3-B
+    } else if (tX > tY) { den = tY + 1; beta = lX - lY; }                    // Case 4-A
+    else if (lX > lY) { den = (uint64_t)y1 + 1; beta = lX - lY - 1; }        // Case 4-B
+    else { num = 1; den = 1; beta = 0; }                                      // Case 4-C: (1, 0)
+    if (den == 1) {
+        alpha = (uint32_t)num;  // 4-C, or a divisor of 1 (then num < 2^32, L133)
+        return;
+    }
+    bool near;
+    uint32_t qhi;
+    uint32_t q = div_floor_est(num, den, near, qhi);
+    if (near) q = div_floor_fix(num, den, qhi);
+    alpha = q;  // < 2^32 outside Case 1 (L133); the bound alpha*D^beta <= X div Y is L123's
 }
 
 // One iteration's update of X (X >= Y > 0 odd, lX >= 3): beta = 0 -> X <- rshift(X - alpha*Y) with alpha
@@ -162,6 +181,83 @@ __device__ __forceinline__ bool s_update(SOp X, int lX, SOp Y, uint32_t alpha, i
     }
     s_rshift(X, lX);
     return true;
+}
+
+// Four limbs k..k+3 of the fused pass X <- rshift(X - alpha*Y) (W1, L233) in one PTX block:
+// the product carry h rides in the 64-bit addend of mad.wide (IMAD.WIDE + IADD3 + IMAD.X),
+// the borrow in the CC flag of a subc.cc chain, saved between chunks in b (0 or ~0u: one
+// sub.cc to restore it, one subc to save it), and the funnel shift produces the words k-1..k+2
+// of the shifted result from (zp, z_k..z_{k+3}).  (A two-borrow-chain form -- independent
+// products, a shorter dependency per limb -- measured 7.9 -> 8.3 ms on cfg7: not taken.)
+__device__ __forceinline__ void s_chunk4(const uint32_t (&x)[4], const uint32_t (&y)[4], uint32_t alpha, uint32_t r,
+                                         uint32_t &h, uint32_t &b, uint32_t &zp, uint32_t (&o)[4]) {
+    asm("{\n\t.reg .u32 lo, hi, z0, z1, z2, z3, t;\n\t.reg .u64 p, q;\n\t"
+        "sub.cc.u32 t, 0, %6;\n\t"
+        "mov.b64 q, {%5, 0};\n\tmad.wide.u32 p, %15, %11, q;\n\tmov.b64 {lo, hi}, p;\n\tsubc.cc.u32 z0, %7, lo;\n\t"
+        "mov.b64 q, {hi, 0};\n\tmad.wide.u32 p, %15, %12, q;\n\tmov.b64 {lo, hi}, p;\n\tsubc.cc.u32 z1, %8, lo;\n\t"
+        "mov.b64 q, {hi, 0};\n\tmad.wide.u32 p, %15, %13, q;\n\tmov.b64 {lo, hi}, p;\n\tsubc.cc.u32 z2, %9, lo;\n\t"
+        "mov.b64 q, {hi, 0};\n\tmad.wide.u32 p, %15, %14, q;\n\tmov.b64 {lo, hi}, p;\n\tsubc.cc.u32 z3, %10, lo;\n\t"
+        "subc.u32 %6, 0, 0;\n\t"
+        "mov.u32 %5, hi;\n\t"
+        "shf.r.wrap.b32 %0, %4, z0, %16;\n\tshf.r.wrap.b32 %1, z0, z1, %16;\n\t"
+        "shf.r.wrap.b32 %2, z1, z2, %16;\n\tshf.r.wrap.b32 %3, z2, z3, %16;\n\t"
+        "mov.u32 %4, z3;\n\t}"
+        : "=r"(o[0]), "=r"(o[1]), "=r"(o[2]), "=r"(o[3]), "+r"(zp), "+r"(h), "+r"(b)
+        : "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(y[0]), "r"(y[1]), "r"(y[2]), "r"(y[3]), "r"(alpha),
+          "r"(r));
+}
+
+// The beta = 0 update of the lockstep loop (s_euclid_ls): the same X <- rshift(X - alpha*Y) as
+// s_update, but the pass runs to the warp-uniform bound L (the longest running lane's lX; the
+// words of a shorter lane at and above its lX are zero and stay zero, since X - alpha*Y >= 0
+// leaves no borrow or carry out of word lX - 1), in chunks of 4 limbs, so every running lane
+// executes the same straight-line code, and it is software-pipelined: chunk c + 1 is loaded
+// before chunk c is computed and stored (X and Y are different buffers and a store only
+// writes a word already read).  Chunks may run past L into the SM_PAD zero words that pad
+// every operand buffer (they read zeros and write zeros).  The rare routes (beta > 0, rshift
+// by >= 32 bits) fall back to s_update.
+__device__ __forceinline__ bool s_update_ls(SOp X, int lX, SOp Y, uint32_t alpha, int beta, int L) {
+    if (beta != 0) return s_update(X, lX, Y, alpha, beta);
+    alpha -= ~alpha & 1u;  // alpha is odd (L107)
+    const uint32_t x0 = X[0], y0 = Y[0];
+    uint64_t p = (uint64_t)alpha * y0;
+    uint32_t h = (uint32_t)(p >> 32);
+    uint32_t zp = x0 - (uint32_t)p;
+    uint32_t b = x0 < (uint32_t)p ? ~0u : 0u;
+    if (zp == 0u) return s_update(X, lX, Y, alpha, 0);  // rshift by >= 32 bits: the plain route
+    const uint32_t r = __clz(__brev(zp));
+    uint32_t xa[4], ya[4], xb[4], yb[4], o[4];
+    const uint32_t *px = X.p, *py = Y.p;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        xa[i] = px[(1 + i) * 32];
+        ya[i] = py[(1 + i) * 32];
+    }
+    int k0 = 1;
+    for (;;) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {  // prefetch the next chunk
+            xb[i] = px[(k0 + 4 + i) * 32];
+            yb[i] = py[(k0 + 4 + i) * 32];
+        }
+        s_chunk4(xa, ya, alpha, r, h, b, zp, o);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) X[k0 - 1 + i] = o[i];
+        k0 += 4;
+        if (k0 >= L) break;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            xa[i] = px[(k0 + 4 + i) * 32];
+            ya[i] = py[(k0 + 4 + i) * 32];
+        }
+        s_chunk4(xb, yb, alpha, r, h, b, zp, o);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) X[k0 - 1 + i] = o[i];
+        k0 += 4;
+        if (k0 >= L) break;
+    }
+    X[k0 - 1] = zp >> r;  // top word of the last chunk (k0 - 1 >= L - 1; a zero word if above L - 1)
+    return false;
 }
 
 // Binary Euclid step on one operand T (L57): T <- (T - c*Y) / 2, c in {0, 1}, lT words.
@@ -225,6 +321,41 @@ __device__ __forceinline__ void s_euclid(SOp &X, SOp &Y, int &lX, uint64_t &tX, 
             SOp t = X; X = Y; Y = t;
             int tl = lX; lX = lY; lY = tl;
             uint64_t tt = tX; tX = tY; tY = tt;
+        }
+    }
+}
+
+// The Approximate Euclidean loop (ALG_APPROX) in warp lockstep: every lane of the warp calls
+// it (`live` = the lane has a pair to run); each trip is one iteration of every still-running
+// lane, with the fused pass bounded by the longest running operand (s_update_ls).  Same
+// arithmetic, counters and results as s_euclid, lane for lane.
+template <bool EXACT, bool STATS>
+__device__ __forceinline__ void s_euclid_ls(SOp &X, SOp &Y, int &lX, uint64_t &tX, int &lY, uint64_t &tY, int half,
+                                            bool live, uint32_t &iters, uint32_t &rare, uint32_t &limbs,
+                                            uint32_t &betapos) {
+    for (;;) {
+        bool run = live && (EXACT ? ((lY >= 1) & (lX >= 3)) : s_rsa_run(lY, tY, half));
+        if (!__any_sync(0xffffffffu, run)) break;
+        const int L = (int)__reduce_max_sync(0xffffffffu, run ? (unsigned)lX : 0u);
+        live = run;
+        if (run) {
+            uint32_t alpha;
+            int beta;
+            s_approx(lX, tX, lY, tY, alpha, beta);
+            if (STATS) {
+                ++iters;
+                limbs += lX;
+                betapos += beta > 0;
+            }
+            bool rr = s_update_ls(X, lX, Y, alpha, beta, L);
+            if (STATS) rare += rr;
+            lX = s_len(X, lX);
+            tX = s_top(X, lX);
+            if (s_cmp(X, lX, tX, Y, lY, tY) < 0) {  // "if (X < Y) swap(X, Y)": a pointer swap (L227)
+                SOp t = X; X = Y; Y = t;
+                int tl = lX; lX = lY; lY = tl;
+                uint64_t tt = tX; tX = tY; tY = tt;
+            }
         }
     }
 }

@@ -205,7 +205,45 @@ CFG2_PAIRS = 1 << 20
 
 
 def config_moduli(k: int, nthreads: int | None = None) -> ModuliSet:
+    if k == 8:
+        return moduli_cofactors(seed=2015 + k, **CONFIG8)
     return moduli(seed=2015 + k, nthreads=nthreads, **CONFIGS[k])
+
+
+def random_cofactors(count: int, pbits: int, seed: int) -> np.ndarray:
+    """count seeded random ODD pbits-bit integers with the top two bits set (the size
+    profile of OpenSSL primes, without the primality test), uint32[count, pbits/32]."""
+    rng = np.random.Generator(np.random.Philox(key=seed))
+    P = rng.integers(0, 1 << 32, size=(count, pbits // 32), dtype=np.uint64).astype(np.uint32)
+    P[:, 0] |= 1
+    P[:, -1] |= 0xC0000000
+    return P
+
+
+def moduli_cofactors(m: int, bits: int, seed: int, n_planted_pairs: int = 0) -> ModuliSet:
+    """The paper's 4096-bit Table V workload size (all pairs of 16,384
+    moduli) with fast inputs: n_i = p_i * q_i from random odd bits/2-bit cofactors (top two
+    bits set) instead of primes -- 32,768 2048-bit primes take ~40 min to draw on 16 cores.
+    The Euclid statistics depend only on the operand sizes (same s, same top-bit profile).
+    Planted pairs (a, b) share p_a, so p_a divides gcd(n_a, n_b); a non-planted pair would
+    need a common factor of >= bits/2 bits between random products (negligible).  `truth`
+    lists the planted (a, b, None): the gcd value is checked by divisibility, not stored."""
+    P = random_cofactors(2 * m, bits // 2, seed)
+    p, q = P[0::2].copy(), P[1::2].copy()
+    rng = np.random.Generator(np.random.Philox(key=seed + 1))
+    perm = [int(x) for x in rng.permutation(m)]
+    groups = []
+    for g in range(n_planted_pairs):
+        a, b = sorted(perm[2 * g:2 * g + 2])
+        p[b] = p[a]
+        groups.append((a, b))
+    N = multiply(p, q)
+    return ModuliSet(bits, N, np.stack([p, q], axis=1).reshape(2 * m, -1), groups, [],
+                     sorted((a, b, None) for a, b in groups))
+
+
+# cfg8: 16,384 x 4096-bit moduli, all 134,209,536 pairs (the paper's Table V 4096-bit size; N1)
+CONFIG8 = dict(m=16384, bits=4096, n_planted_pairs=8)
 
 
 def pair_indices(n: int, count: int) -> tuple[np.ndarray, np.ndarray]:

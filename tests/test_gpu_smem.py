@@ -110,6 +110,35 @@ def test_table4_4096_means(bg):
         assert abs(x.mean() - paper) < 4 * se + 0.5, (x.mean(), paper, se)
 
 
+def test_beta_positive_rate_4096(bg):
+    """at 4096 bits, approx() returns beta != 0 in 1191 of 201,277,617,364
+    calls (non-terminate runs, reading 19).  2^18 pairs of random odd 4096-bit
+    operands with the top two bits set (the size profile of the paper's moduli), exact
+    mode = non-terminate: the GPU's beta > 0 count (counter 7 of the shared-memory
+    kernel) equals, event for event, the count of the C implementation of the paper's
+    algorithm (oracle/approx_euclid.c) on the same pairs, and the rate is consistent with
+    the paper's 5.9e-9 (a Poisson interval around the expected ~2.4 events)."""
+    import os
+    m = 1 << 18
+    rng = np.random.default_rng(4253)
+    X = rng.integers(0, 1 << 32, size=(2 * m, 128), dtype=np.uint64).astype(np.uint32)
+    X[:, 0] |= 1
+    X[:, 127] |= 0xC0000000
+    A, B = X[:m], X[m:]
+    G, it, st = _pairs_device(bg, A, B, 4096, bg.MODE_EXACT, 0)
+    calls, beta_gpu = int(st[2]), int(st[7])
+    k = np.arange(m, dtype=np.uint64)
+    Gc, itc, ctr = oracle.approx_index_pairs(X, k, k + m, 4096, early=False, nthreads=os.cpu_count() or 1)
+    assert np.array_equal(G, Gc) and np.array_equal(it, itc)
+    assert calls == ctr[0] == int(it.sum())
+    assert beta_gpu == ctr[2]
+    expect = calls * 1191 / 201_277_617_364
+    assert 1400 < calls / m < 1650  # ~1523 iterations per non-terminate 4096-bit GCD (Table IV, reading 19)
+    assert beta_gpu <= expect + 6 * math.sqrt(expect) + 6, (beta_gpu, expect)
+    print(f"beta>0: {beta_gpu} of {calls} approx calls ({beta_gpu / calls:.3g}; paper 1191/2.01e11 = 5.92e-9; "
+          f"expected {expect:.1f})")
+
+
 # ------------------------------------------------------- 4096-bit all pairs
 def test_all_pairs_4096(bg, ms4096):
     hits = bg.bulkgcd_all_pairs(ms4096.N, 4096)

@@ -1,0 +1,4 @@
+O=gpurun_out/r2j; mkdir -p $O
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:allpairs_smem -c 1 -o $O/smem_src python tools/prof_allpairs.py 512 4096 1 > $O/ncu.log 2>&1
+ncu -i $O/smem_src.ncu-rep --page source --csv --print-source sass > $O/smem_src.csv 2>/dev/null
+ncu -i $O/smem_src.ncu-rep --page raw --csv > $O/smem_raw.csv 2>/dev/null
