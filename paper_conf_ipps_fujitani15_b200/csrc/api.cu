@@ -128,9 +128,13 @@ int launch_pairs_smem_alg(const PairsArgs &a, int mode, bool stats, cudaStream_t
     static PerDeviceOnce attr_once;  // dynamic shared memory opt-in, per device
     if (int rc = attr_once.run([]() -> int {
             CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, true, ALG>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, true, false, ALG>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, true, ALG>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(pairs_smem_kernel<W, false, false, ALG>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             return 0;
         }))
         return rc;
@@ -189,7 +193,9 @@ int launch_allpairs_smem_alg(const AllPairsArgs &a, bool stats, cudaStream_t st)
     static PerDeviceOnce attr_once;  // dynamic shared memory opt-in, per device
     if (int rc = attr_once.run([]() -> int {
             CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, true, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, true, ALG>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, false, ALG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(allpairs_smem_kernel<W, false, ALG>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             return 0;
         }))
         return rc;
@@ -228,10 +234,16 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     constexpr int wpc = ApCfg<W>::warps_per_cta;
     uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * ApCfg<W>::blocks, (warps + wpc - 1) / wpc);
     constexpr size_t smem = allpairs_smem_bytes<W>();
-    static PerDeviceOnce attr_once;  // dynamic shared memory opt-in, per device
+    // dynamic shared memory opt-in and the largest shared-memory carveout, per device: the
+    // residency of these kernels is set by their per-warp staging buffers, and with small
+    // CTAs the driver's default carveout can leave room for fewer of them than the
+    // register budget allows
+    static PerDeviceOnce attr_once;
     if (int rc = attr_once.run([]() -> int {
             CK(cudaFuncSetAttribute(allpairs_kernel<W, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(allpairs_kernel<W, true>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             CK(cudaFuncSetAttribute(allpairs_kernel<W, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(allpairs_kernel<W, false>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
             return 0;
         }))
         return rc;

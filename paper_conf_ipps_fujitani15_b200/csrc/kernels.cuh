@@ -564,9 +564,12 @@ struct StageBuf {
 #ifndef BULKGCD_AP_THREADS_NARROW
 #define BULKGCD_AP_THREADS_NARROW 32
 #endif
+#ifndef BULKGCD_AP_THREADS_W64
+#define BULKGCD_AP_THREADS_W64 128
+#endif
 template <int W>
 struct ApCfg {
-    static constexpr int threads = W <= 32 ? BULKGCD_AP_THREADS_NARROW : 128;
+    static constexpr int threads = W <= 32 ? BULKGCD_AP_THREADS_NARROW : BULKGCD_AP_THREADS_W64;
     static constexpr int warps_per_cta = threads / 32;
     static constexpr int warps = Occ<W>::warps;  // resident warps per SM (register budget)
     static constexpr int blocks = warps / warps_per_cta > 0 ? warps / warps_per_cta : 1;
