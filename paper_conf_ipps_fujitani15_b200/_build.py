@@ -14,7 +14,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 SO = os.path.join(PKG, "libbulkgcd.so")
 SOURCES = ["api.cu"]
-HEADERS = ["kernels.cuh", "euclid.cuh", "smem_euclid.cuh", "duff_pass.cuh", "factor.cuh", "gen_duff.py"]
+HEADERS = ["kernels.cuh", "euclid.cuh", "smem_euclid.cuh", "hybrid_euclid.cuh", "duff_pass.cuh", "factor.cuh", "gen_duff.py"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 NVCC_FLAGS = [

@@ -223,7 +223,27 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
     if (c1 <= c0) return 0;
     AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
     if constexpr (W >= 128) {
-        return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
+        // the 4096-bit product path: the hybrid kernel (A in registers, B in shared memory);
+        // BULKGCD_FLAG_SMEM and the comparison algorithms keep the shared-memory kernels
+        if ((flags & BULKGCD_FLAG_SMEM) || (flags & BULKGCD_FLAG_ALGO_MASK))
+            return launch_allpairs_smem<W>(a, (flags & BULKGCD_FLAG_STATS) != 0, flags, st);
+        constexpr size_t smem = hybrid_smem_bytes<W>();
+        static PerDeviceOnce attr_once;
+        if (int rc = attr_once.run([]() -> int {
+                CK(cudaFuncSetAttribute(allpairs_hybrid_kernel<W, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                CK(cudaFuncSetAttribute(allpairs_hybrid_kernel<W, true>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+                CK(cudaFuncSetAttribute(allpairs_hybrid_kernel<W, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                CK(cudaFuncSetAttribute(allpairs_hybrid_kernel<W, false>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+                return 0;
+            }))
+            return rc;
+        uint64_t warps = c1 - c0;
+        constexpr int wpc = HY_THREADS / 32;
+        uint64_t grid = std::min<uint64_t>((uint64_t)sm_count() * HY_BLOCKS, (warps + wpc - 1) / wpc);
+        if (flags & BULKGCD_FLAG_STATS) allpairs_hybrid_kernel<W, true><<<(unsigned)grid, HY_THREADS, smem, st>>>(a);
+        else allpairs_hybrid_kernel<W, false><<<(unsigned)grid, HY_THREADS, smem, st>>>(a);
+        CK(cudaGetLastError());
+        return 0;
     } else {
     // the comparison algorithms run on the shared-memory kernels (per-lane pointer swap,
     // the paper's own design): (D) there measures 661 ms on cfg3 against 1,235 ms on

@@ -244,6 +244,89 @@ def emit_cmpl(W: int, G: int, ones: bool) -> str:
     return "\n".join(o)
 
 
+def emit_hybrid(W: int, G: int, side: str) -> str:
+    """Hybrid passes of the 4096-bit all-pairs kernel (kernels.cuh allpairs_hybrid_kernel):
+    operand A lives in registers (top-aligned like every register kernel: word i at
+    register s + i), operand B in shared memory, least significant word first, one row of
+    32 lanes per word; with base = (B's row 0 address) - 128 s, B's word at register
+    position k is at [base + 128 k] -- a static immediate per limb, and realigning A
+    (s += 1) is a change of base, B never moves.
+      side "A": A <- rshift(A - alpha*B), B read from shared memory;
+      side "B": B <- rshift(B - alpha*A), B read and written in shared memory.
+    Split form per limb (IMAD.WIDE carry addend, subc.cc borrow chain, funnel shift), G-limb
+    blocks behind a brx.idx jump table on s, like emit().
+
+    Operands: %0 = r (out), %1 = z_s (out), %2..%(W+1) = A[k] (side A: in/out, side B: in),
+    %(W+2) = alpha, %(W+3) = s, %(W+4) = base (32-bit shared address)."""
+    av = lambda k: "%%%d" % (2 + k)
+    al = "%%%d" % (W + 2)
+    sa = "%%%d" % (W + 3)
+    ba = "%%%d" % (W + 4)
+    K = lambda k: 128 * k
+    a = ["{", ".reg .u32 zp, z, lo, hi, t, v, w;", ".reg .u64 p, q;", ".reg .pred pe;",
+         "setp.ge.s32 pe, %s, 0;" % sa,
+         "ts: .branchtargets %s;" % ", ".join("E%d" % k for k in range(W)),
+         "brx.idx %s, ts;" % sa]
+
+    def ldv(k):  # the shared-memory operand's word at register position k -> v
+        return ["ld.shared.u32 v, [%s+%d];" % (ba, K(k))]
+
+    def limb(k):
+        out = ldv(k) + ["mov.b64 q, {hi, 0};"]
+        if side == "A":
+            out += ["mad.wide.u32 p, %s, v, q;" % al, "mov.b64 {lo, hi}, p;",
+                    "subc.cc.u32 z, %s, lo;" % av(k),
+                    "shf.r.wrap.b32 %s, zp, z, %%0;" % av(k - 1)]
+        else:
+            out += ["mad.wide.u32 p, %s, %s, q;" % (al, av(k)), "mov.b64 {lo, hi}, p;",
+                    "subc.cc.u32 z, v, lo;",
+                    "shf.r.wrap.b32 w, zp, z, %0;",
+                    "st.shared.u32 [%s+%d], w;" % (ba, K(k - 1))]
+        return out + ["mov.u32 zp, z;"]
+
+    for k in range(W):
+        e = min((k // G + 1) * G, W)
+        nxt = "B%d" % e if e < W else "TOP"
+        a += ["E%d:" % k] + ldv(k)
+        if side == "A":
+            a += ["mul.wide.u32 p, %s, v;" % al, "mov.b64 {lo, hi}, p;", "sub.cc.u32 zp, %s, lo;" % av(k)]
+        else:
+            a += ["mul.wide.u32 p, %s, %s;" % (al, av(k)), "mov.b64 {lo, hi}, p;", "sub.cc.u32 zp, v, lo;"]
+        a += ["mov.u32 %1, zp;", "brev.b32 t, zp;", "clz.b32 %0, t;"]
+        for j in range(k + 1, e):
+            a += limb(j)
+        a.append("@pe bra %s;" % nxt)
+    a.append("bra.uni TOP;")
+    for k in range(1, W):
+        if k % G == 0:
+            a.append("B%d:" % k)
+        a += limb(k)
+    if side == "A":
+        a += ["TOP:", "shf.r.wrap.b32 %s, zp, 0, %%0;" % av(W - 1), "}"]
+    else:
+        a += ["TOP:", "shf.r.wrap.b32 w, zp, 0, %0;", "st.shared.u32 [%s+%d], w;" % (ba, K(W - 1)), "}"]
+    body = "\\n\\t".join(x.replace('"', '\\"') for x in a)
+    if side == "A":
+        outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(A[%d])' % k for k in range(W)]
+        ins = ['"r"(alpha)', '"r"(s)', '"r"(base)']
+        sig = "uint32_t (&A)[%d]" % W
+    else:
+        outs = ['"=r"(r)', '"=r"(zs)']
+        ins = ['"r"(A[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)', '"r"(base)']
+        sig = "uint32_t (&A)[%d]" % W  # read only (asm inputs)
+    o = ["template <>",
+         "__device__ __forceinline__ uint32_t duff_hpass<%d, %d, '%s'>(%s, uint32_t alpha, int s, uint32_t base, "
+         "uint32_t &r) {" % (W, G, side, sig),
+         "  uint32_t zs;",
+         '  asm volatile("%s"' % body,
+         "      : %s" % ", ".join(outs),
+         "      : %s" % ", ".join(ins),
+         '      : "memory");',
+         "  return zs;",
+         "}"]
+    return "\n".join(o)
+
+
 def main():
     import sys
     form = sys.argv[1] if len(sys.argv) > 1 else os.environ.get("BULKGCD_PASS_FORM", "split")
@@ -289,6 +372,16 @@ def main():
         "__device__ __forceinline__ uint32_t duff_cpass(uint32_t (&X)[W], const uint32_t (&Y)[W], uint32_t alpha,",
         "                                               uint32_t cin, int s, uint32_t &r);",
         "",
+    ]
+    GH = int(os.environ.get("BULKGCD_PASS_G_HYBRID", "4"))
+    parts += [
+        "// Hybrid passes (emit_hybrid): A in registers, B in shared memory at [base + 128 k].",
+        "template <int W, int G, char SIDE, class AR>",
+        "__device__ __forceinline__ uint32_t duff_hpass(AR &A, uint32_t alpha, int s, uint32_t base, uint32_t &r);",
+        "constexpr int PASS_G_HYBRID = %d;" % GH,
+        "",
+        emit_hybrid(128, GH, "A"), "",
+        emit_hybrid(128, GH, "B"), "",
     ]
     for W in WIDTHS:
         gw = G64 if W >= 64 else (G16 if W <= 16 else G)

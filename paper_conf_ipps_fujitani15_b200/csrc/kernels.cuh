@@ -866,3 +866,5 @@ __global__ void __launch_bounds__(SM_THREADS) allpairs_smem_kernel(AllPairsArgs 
 }
 
 }  // namespace bulkgcd
+
+#include "hybrid_euclid.cuh"  // the 4096-bit all-pairs kernel (one operand in registers, one in shared memory)

@@ -149,6 +149,35 @@ def test_all_pairs_4096(bg, ms4096):
     assert got == oracle.cofactors(ms4096.N, ms4096.truth)
 
 
+def test_all_pairs_4096_hybrid_equals_smem_kernel(bg, ms4096):
+    """The 4096-bit all-pairs product path is the hybrid kernel (A in registers, B in
+    shared memory, hybrid_euclid.cuh); BULKGCD_FLAG_SMEM forces the shared-memory kernel.
+    Both run the same algorithm with the exact-floor approx(), so they must agree on the
+    hit set, on the total iteration count and on the limb-steps (M2's units), and the
+    totals must equal the paper-algorithm model's over every pair."""
+    W, n = 128, ms4096.m
+    dev = torch.device("cuda")
+    dN = torch.from_numpy(ms4096.N.view(np.int32)).to(dev)
+    dB = torch.empty(bg.bulkgcd_blocked_words(n, 4096), dtype=torch.int32, device=dev)
+    bg.bulkgcd_layout_blocked(dN, dB, n, 4096)
+    total = bg.bulkgcd_cohort_count(n)
+    out = {}
+    for name, fl in (("hybrid", 0), ("smem", bg.FLAG_SMEM)):
+        dH = torch.zeros(64 * (2 + W), dtype=torch.int32, device=dev)
+        dC = torch.zeros(8, dtype=torch.int64, device=dev)
+        bg.bulkgcd_all_pairs_band(dN, dB, n, 4096, 0, total, dH, 64, dC, bg.FLAG_STATS | fl)
+        torch.cuda.synchronize()
+        c = dC.cpu().numpy()
+        rec = dH.cpu().numpy().view(np.uint32).reshape(-1, 2 + W)[:int(c[0])]
+        out[name] = (sorted((int(r[0]), int(r[1]), synth.to_int(r[2:])) for r in rec), int(c[2]), int(c[4]))
+    assert out["hybrid"] == out["smem"]
+    N = synth.ints(ms4096.N)
+    tr = [am.gcd_rsa(N[i], N[j], 4096) for i in range(n) for j in range(i + 1, n)]
+    assert out["hybrid"][0] == ms4096.truth
+    assert out["hybrid"][1] == sum(t.iterations for t in tr)
+    assert out["hybrid"][2] == sum(t.limb_steps for t in tr)
+
+
 # ---------------------------- the smem kernels forced at register widths
 @pytest.mark.parametrize("bits", [512, 1024, 2048])
 def test_smem_flag_matches_register_kernels(bg, bits):
