@@ -556,7 +556,7 @@ def main():
         iters, limbs, slots, passw, betapos = (int(x) for x in tt)
     # SIMT efficiencies of the lockstep register kernels (the smem kernels run lanes independently)
     eff = {"lane_efficiency": iters / slots if slots else None,
-           "pass_word_efficiency": limbs / passw if passw else None} if (W < 128 and args.algo == "E") else None
+           "pass_word_efficiency": limbs / passw if passw else None} if args.algo == "E" else None
 
     k0 = torch.cuda.Event(enable_timing=True)
     k1 = torch.cuda.Event(enable_timing=True)
@@ -647,19 +647,20 @@ def main():
             "data": "synthetic",
             "config": {"workload": WORKLOADS[args.workload],
                        "n": n, "bits": bits, "pairs": pairs, "mode": "rsa-early-terminate",
-                       "algorithm": {"E": "approximate-euclid (" + ("register" if W < 128 else "shared-memory") + "-resident)",
+                       "algorithm": {"E": "approximate-euclid (" + ("register-resident" if W < 128 else
+                                                                     "hybrid: one operand in registers, one in shared memory") + ")",
                                      "D": "fast-binary-euclid (ablation, smem)",
                                      "C": "binary-euclid (ablation, smem)"}[args.algo],
                        "parallelism": f"row-band x{world}" + (" + NCCL hit all-gather" if world > 1 else ""),
                        "l2": "flushed before every step (256 MiB write); inputs 2 MiB",
                        "ns_per_gcd": step_total_ms / args.steps * 1e6 / pairs,
                        "iterations_per_gcd": iters / pairs, "limb_steps_per_gcd": limbs / pairs,
-                       "beta_pos_iterations": betapos if W >= 128 else None,
+
                        "ms_per_step_median": statistics.median(step_ms), "ms_per_step_min": min(step_ms),
                        "hits_ok": bool(ok), "hits": len(found), "wall_s": t_wall},
             # per-GPU kernel throughput: each rank runs 1/world of the work
             "roofline": roofline(limbs / world, iters / world, pairs / world, kern_s, sms,
-                                 (f"allpairs_kernel<{W}>" if W < 128 else f"allpairs_smem_kernel<{W}>")
+                                 (f"allpairs_kernel<{W}>" if W < 128 else f"allpairs_hybrid_kernel<{W}>")
                                  if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
                                  kern_total_ms / step_total_ms, _traffic(args.workload), eff),
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,

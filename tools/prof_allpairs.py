@@ -9,11 +9,17 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_ipps_fujitani15_b200 as bg  # noqa: E402
 import synth  # noqa: E402
 
-n = int(sys.argv[1]) if len(sys.argv) > 1 else 2048
-bits = int(sys.argv[2]) if len(sys.argv) > 2 else 1024
-reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
+# python tools/prof_allpairs.py N BITS [REPS]  (random moduli)  |  python tools/prof_allpairs.py cfgK [REPS]
+if len(sys.argv) > 1 and sys.argv[1].startswith("cfg"):
+    ms = synth.config_moduli(int(sys.argv[1][3:]))
+    n, bits = ms.m, ms.bits
+    reps = int(sys.argv[2]) if len(sys.argv) > 2 else 1
+else:
+    n = int(sys.argv[1]) if len(sys.argv) > 1 else 2048
+    bits = int(sys.argv[2]) if len(sys.argv) > 2 else 1024
+    reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
+    ms = synth.moduli(n, bits, seed=5, n_planted_pairs=2)
 W = bits // 32
-ms = synth.moduli(n, bits, seed=5, n_planted_pairs=2)
 dev = torch.device("cuda")
 dN = torch.from_numpy(ms.N.view(np.int32)).to(dev)
 dB = torch.empty(bg.bulkgcd_blocked_words(n, bits), dtype=torch.int32, device=dev)
