@@ -18,11 +18,32 @@ Per limb k of the body (SASS on sm_100a):
     SHF.R.W        X[k-1] = funnel(z_{k-1}, z_k, r)  (rshift, L37)
 plus the register-pair shuffle ptxas needs for the 64-bit addend.
 
+Limb forms (template argument F of duff_pass, `form_code`):
+    split  IMAD.WIDE.U32 (zero addend), IADD3 carry-add, IMAD.X, IADD3.X, SHF.R.W:
+           three ALU-pipe and two FMA-pipe instructions per limb;
+    wide   IMAD.WIDE.U32 with the 64-bit addend {h, 0} (PTX mul.wide + shr + add.s64),
+           IMAD.MOV (pair shuffle), IADD3.X, SHF.R.W: the carry-add moves to the FMA pipe;
+    mixM   every M-th limb split, the others wide.  The all-pairs kernel's ALU pipe is the
+           busiest unit (ncu: 72.7 % against 55 % fmaheavy on cfg3), so mix2 balances the two:
+           cfg3 240.9 -> 233.3 ms, cfg6 82.0 -> 80.7 ms (wide 238.7, mix3 237.7, mix4 238.6).
+
 Run:  python gen_duff.py  (writes duff_pass.cuh next to this file)
 """
 import os
 
 WIDTHS = (16, 32, 64)
+
+
+def form_code(form: str) -> int:
+    """duff_pass's third template argument: 0 split, 1 wide, M >= 2 mixM, 100 two-chain."""
+    if form == "split":
+        return 0
+    if form == "wide":
+        return 1
+    if form == "two":
+        return 100
+    assert form.startswith("mix") and int(form[3:]) >= 2, form
+    return int(form[3:])
 
 
 def emit(W: int, form: str = "split", G: int = 1) -> str:
@@ -38,6 +59,7 @@ def emit(W: int, form: str = "split", G: int = 1) -> str:
     Operands: %0 = r (out), %1 = z_s (out), %2..%(W+1) = X[k] (in/out),
     %(W+2)..%(2W+1) = Y[k], %(2W+2) = alpha, %(2W+3) = s.
     """
+    FCODE = form_code(form)
     xa = lambda k: "%%%d" % (2 + k)
     ya = lambda k: "%%%d" % (W + 2 + k)
     al = "%%%d" % (2 * W + 2)
@@ -47,11 +69,13 @@ def emit(W: int, form: str = "split", G: int = 1) -> str:
          "ts: .branchtargets %s;" % ", ".join("E%d" % k for k in range(W)),
          "brx.idx %s, ts;" % sa]
     def limb(k):  # body limb k >= 1: product with carry, borrow chain, funnel shift into X[k-1]
-        if form == "wide":  # 64-bit addend: IMAD.WIDE.U32 + pair shuffle (product chain on the FMA pipe)
+        # "mixM": every M-th limb split, the rest wide (balances the ALU and FMA pipes)
+        wide = form == "wide" or (form.startswith("mix") and k % int(form[3:]) != 0)
+        if wide:  # 64-bit addend: IMAD.WIDE.U32 + pair shuffle (product chain on the FMA pipe)
             out = ["mul.wide.u32 m, %s, %s;" % (al, ya(k)),
                    "shr.u64 q, p, 32;",
                    "add.s64 p, m, q;",
-                   "cvt.u32.u64 lo, p;"]
+                   "mov.b64 {lo, hi}, p;"]
         else:  # split: IMAD.WIDE + 32-bit add-with-carry of the high half
             out = ["mov.b64 q, {hi, 0};",
                    "mad.wide.u32 p, %s, %s, q;" % (al, ya(k)),
@@ -86,8 +110,8 @@ def emit(W: int, form: str = "split", G: int = 1) -> str:
     outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(X[%d])' % k for k in range(W)]
     ins = ['"r"(Y[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)']
     o = ["template <>",
-         "__device__ __forceinline__ uint32_t duff_pass<%d, %d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
-         "uint32_t alpha, int s, uint32_t &r) {" % (W, G, W, W),
+         "__device__ __forceinline__ uint32_t duff_pass<%d, %d, %d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
+         "uint32_t alpha, int s, uint32_t &r) {" % (W, G, FCODE, W, W),
          "  uint32_t zs;",
          '  asm volatile("%s"' % body,
          "      : %s" % ", ".join(outs),
@@ -103,6 +127,7 @@ def emit_two(W: int, G: int) -> str:
     (tools/limbmix.cu: no carry-add / IMAD.X per limb; 9.5 -> 8.9 SMSP-cycles per
     limb in isolation at G = 8).  The borrows cross block boundaries through two
     registers (save: subc 0,0 -> 0 or -1; restore: sub.cc 0, b)."""
+    FCODE = form_code("two")
     xa = lambda k: "%%%d" % (2 + k)
     ya = lambda k: "%%%d" % (W + 2 + k)
     al = "%%%d" % (2 * W + 2)
@@ -169,8 +194,8 @@ def emit_two(W: int, G: int) -> str:
     outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(X[%d])' % k for k in range(W)]
     ins = ['"r"(Y[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)']
     o = ["template <>",
-         "__device__ __forceinline__ uint32_t duff_pass<%d, %d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
-         "uint32_t alpha, int s, uint32_t &r) {" % (W, G, W, W),
+         "__device__ __forceinline__ uint32_t duff_pass<%d, %d, %d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
+         "uint32_t alpha, int s, uint32_t &r) {" % (W, G, FCODE, W, W),
          "  uint32_t zs;",
          '  asm volatile("%s"' % body,
          "      : %s" % ", ".join(outs),
@@ -329,10 +354,15 @@ def emit_hybrid(W: int, G: int, side: str) -> str:
 
 def main():
     import sys
-    form = sys.argv[1] if len(sys.argv) > 1 else os.environ.get("BULKGCD_PASS_FORM", "split")
-    G = int(os.environ.get("BULKGCD_PASS_G", "4"))
-    if form == "two":
-        G = int(os.environ.get("BULKGCD_PASS_G", "8"))
+    # Pass form per kernel family (measured on cfg3 / 2^20 1024-bit pairs, tools/ab_cfg3.sh):
+    #   all-pairs + RSA-mode pairs, W <= 32: mix2 (every other limb with the 64-bit IMAD.WIDE addend:
+    #     half the limbs move their carry-add from the ALU to the FMA pipe): cfg3 240.9 -> 234.2 ms,
+    #     RSA pairs 2.73 -> 2.69 ms (wide 238.7 / 2.82, mix4 238.6 / 2.80);
+    #   exact-mode pairs: split (mix2 3.85 -> 3.94 ms);  W = 64: split (all pairs use the complement form).
+    form = sys.argv[1] if len(sys.argv) > 1 else os.environ.get("BULKGCD_PASS_FORM", "mix2")
+    form64 = os.environ.get("BULKGCD_PASS_FORM64", "split")
+    formx = os.environ.get("BULKGCD_PASS_FORM_EXACT", "split")
+    G = int(os.environ.get("BULKGCD_PASS_G", "8" if form == "two" else "4"))
     # Exact-mode pairs kernel: G = 2 (cfg2 2^20 exact pairs 4.20 -> 3.87 ms; its larger
     # code -- Case-1 tail, L41 normalisation -- misses the i-cache at G = 4).  G = 2 for
     # the all-pairs kernel costs 246.7 -> 250.7 ms on cfg3, G = 8: 247.3 ms (exact 4.99).
@@ -341,6 +371,7 @@ def main():
     G64 = int(os.environ.get("BULKGCD_PASS_G64", "2"))  # W = 64 has its own knob
     G16 = int(os.environ.get("BULKGCD_PASS_G16", str(G)))  # W = 16 at G = 2: cfg6 82.6 -> 83.4 ms (stays 4)
     here = os.path.dirname(os.path.abspath(__file__))
+    fw = lambda W: form64 if W >= 64 else form
     parts = [
         "// GENERATED by gen_duff.py -- do not edit by hand.",
         "// Fused X <- rshift(X - alpha*Y) limb pass with a computed entry (see gen_duff.py).",
@@ -353,8 +384,9 @@ def main():
         "",
         "// Returns z_s (the lowest word of X - alpha*Y); r = ctz(z_s) (32 if z_s == 0, in which",
         "// case the funnel shifts wrap to 0 and X holds X - alpha*Y unshifted).",
-        "// G = limbs per straight-line block of the chain (one predicated branch per block).",
-        "template <int W, int G>",
+        "// G = limbs per straight-line block of the chain (one predicated branch per block);",
+        "// F = limb form (gen_duff.form_code: 0 split, 1 wide, M >= 2 every M-th limb split, 100 two-chain).",
+        "template <int W, int G, int F>",
         "__device__ __forceinline__ uint32_t duff_pass(uint32_t (&X)[W], const uint32_t (&Y)[W], uint32_t alpha, int s,",
         "                                              uint32_t &r);",
         "",
@@ -362,7 +394,10 @@ def main():
         "// 2^18 2048-bit RSA pairs 2.89 -> 2.81 ms; 8-limb blocks: 1,135 ms)",
         "template <int W>",
         "constexpr int PASS_G = W >= 64 ? %d : (W <= 16 ? %d : %d);" % (G64, G16, G),
+        "template <int W>",
+        "constexpr int PASS_F = W >= 64 ? %d : %d;  // %s / %s" % (form_code(form64), form_code(form), form64, form),
         "constexpr int PASS_G_EXACT = %d;  // exact-mode pairs kernel (smaller code: i-cache)" % GX,
+        "constexpr int PASS_F_EXACT = %d;  // %s" % (form_code(formx), formx),
         "",
     ]
     parts += [
@@ -385,8 +420,8 @@ def main():
     ]
     for W in WIDTHS:
         gw = G64 if W >= 64 else (G16 if W <= 16 else G)
-        for g in sorted({gw, GX}):
-            parts.append(emit_two(W, g) if form == "two" else emit(W, form, g))
+        for g, f in sorted({(gw, fw(W)), (GX, formx)}):
+            parts.append(emit_two(W, g) if f == "two" else emit(W, f, g))
             parts.append("")
         for ones in (True, False):
             parts.append(emit_cmpl(W, gw, ones))

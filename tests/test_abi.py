@@ -96,3 +96,18 @@ def test_cohort_enumeration(bg):
                     assert (i, j) not in pairs
                     pairs.add((i, j))
     assert len(pairs) == n * (n - 1) // 2
+
+
+def test_generated_pass_is_committed(tmp_path):
+    """csrc/duff_pass.cuh is what gen_duff.py emits with the default settings (no tuning
+    variable in the environment changes the production kernels)."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                        "paper_conf_ipps_fujitani15_b200", "csrc")
+    env = {k: v for k, v in os.environ.items() if not k.startswith("BULKGCD_")}
+    env["BULKGCD_DUFF_OUT"] = str(tmp_path / "duff_pass.cuh")
+    subprocess.check_call([sys.executable, os.path.join(here, "gen_duff.py")], env=env)
+    with open(os.path.join(here, "duff_pass.cuh")) as f, open(tmp_path / "duff_pass.cuh") as g:
+        assert f.read() == g.read()
