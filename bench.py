@@ -16,13 +16,14 @@ value   : device-timed (CUDA events, sum over the K steps, max over ranks),
 e2e     : the same metric through the public API with HOST buffers: N = 1:
           bulkgcd_all_pairs() (C ABI: H2D, kernels, D2H, sort); N > 1:
           dist.all_pairs_distributed() per rank.  Host-timed per call.
-roofline: the all-pairs kernel, ALU-pipe bound ("alu"; ncu: the busiest unit):
-          algorithmic ALU-pipe lane-ops per launch (3 per
-          limb-step + 16 per iteration, counted exactly by the kernel's stats
-          pass on the same input) over its CUDA-event duration, against the
-          measured ALU-pipe rate (profiles/r1_pipemix.json) x 32 lanes x SMs x
-          the max SM clock of MEASURED_PEAKS.json; "issue" repeats it for all
-          4 + 16 ops against the measured integer issue ceiling.
+roofline: the hot kernel, integer-issue bound ("alu"):
+          algorithmic integer lane-ops per launch (4 per limb-step + 16 per
+          iteration, counted exactly by the kernel's stats pass on the same
+          input) over its CUDA-event duration, against P_int = SMs x 4 SMSPs x
+          32 lanes x 1 instruction/clk x the max SM clock of MEASURED_PEAKS.json;
+          "alu_pipe" repeats it for the ALU-pipe share against the measured
+          ALU-pipe rate (profiles/r1_pipemix.json); "traffic" is the ncu DRAM
+          bytes per launch of the same build (profiles/r2_ncu_traffic.json).
 cpu_baseline (rank 0, N = 1): the C oracle (Original Euclid, oracle/) on a
           bounded seeded sample of the same pairs, all host cores.
 --impl reference: the oracle as it stands is the reference arm (no reference

@@ -166,7 +166,10 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // pass (B + alpha*A~ + alpha).  The roles alternate strictly, which keeps A complemented;
 // the rare cold-section code that reads the operand registers (fix-ups, the hit sink)
 // sees plain values (A is complemented around it).
-template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, bool CMPL = false>
+// HOIST: approx() for the next iteration is computed at the end of the current one, ahead of
+// its votes and branches (measured: cfg4 851.5 -> 834.6 ms; cfg3 233.3 -> 235.1, 2^20 RSA pairs
+// 2.47 -> 3.07, exact 3.74 -> 3.84 ms: the W = 64 all-pairs kernel only).
+template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, bool CMPL = false, bool HOIST = false>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
@@ -175,6 +178,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
     using CmB = std::integral_constant<int, CMPL ? 2 : 0>;  // ... with B updated
     int s = s0;
     int fix = 0;     // pending fix-up of the last iteration (hot_iter's code)
+    Approx ap;       // approx() for the coming hot iteration
     int resume = 0;  // roles of the next iteration: 0 -> (X, Y) = (A, B), 1 -> (B, A)
     if (CMPL) cmpl_regs<W>(A);
 
@@ -222,12 +226,14 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
             }
         }
         bool full, post, lt;
-        hot_iter<W, EXACT, decltype(cm)::value>(X, Y, lX, tX, lY, tY, s, live, full, post, lt);
+        if (!HOIST) ap = approx_pre<EXACT>(lX, tX, lY, tY);
+        hot_iter<W, EXACT, decltype(cm)::value>(X, Y, lX, tX, lY, tY, s, live, ap, full, post, lt);
         bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
         bool fin = live & !run & !bad;
         bool need = sink.quick_hot(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
+        if (HOIST) ap = approx_pre<EXACT>(lY, tY, lX, tX);  // the next iteration's roles (Y, X), ahead of the votes
         // vote.any with a predicate result: no mask compare on the ALU pipe
         bool any_need = __any_sync(FULL, need), any_top = __any_sync(FULL, top);
         if (any_need) {
@@ -251,6 +257,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
     for (;;) {
         bool more = resume == 0 ? cold(A, B, lA, tA, lB, tB) : cold(B, A, lB, tB, lA, tA);
         if (!more) return;
+        if (HOIST) ap = resume == 0 ? approx_pre<EXACT>(lA, tA, lB, tB) : approx_pre<EXACT>(lB, tB, lA, tA);
         // ONE_ENTRY: resuming on roles (B, A) enters the loop at its second hot
         // iteration, so the pass is inlined twice (once per role assignment) instead of
         // three times.  Measured: RSA pairs 3.30 -> 2.72 ms per 2^20
@@ -698,7 +705,7 @@ __global__ void BULKGCD_AP_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
-        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, allpairs_cmpl<W>()>(
+        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, allpairs_cmpl<W>(), (W >= 64)>(
             A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, 0, iters, nslow, limbs, slots, passw);
         slot ^= 1;
         have = have2;

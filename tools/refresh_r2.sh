@@ -20,6 +20,8 @@ timeout 1800 python tools/ncu_traffic.py $O cfg3 cfg2 cfg4 cfg6 cfg8 > $O/traffi
 ncu -i $O/r2_cfg3.ncu-rep --page source --csv --print-source sass > $O/cfg3_src.csv 2>/dev/null
 ncu -i $O/r2_cfg3.ncu-rep --page raw --csv > $O/cfg3_raw.csv 2>/dev/null
 python tools/ncu_opmix.py $O/cfg3_src.csv > $O/r2_cfg3_opmix.txt 2>&1
+# the reports themselves stay on the box (gpurun copies back at most 64 MiB)
+mkdir -p /tmp/ncu_reps && mv $O/*.ncu-rep /tmp/ncu_reps/ 2>/dev/null; gzip -f $O/cfg3_src.csv
 # compute-sanitizer on the same build
 { echo "# compute-sanitizer on tools/sanitize_run.py (all-pairs at 512/1024/2048/4096 bits incl. the hybrid 4096-bit kernel, exact pairs on rare-path operands, the chunked two-stream host path); build $git_head"
   for t in memcheck racecheck synccheck initcheck; do echo "== $t"; timeout 1200 compute-sanitizer --tool $t python tools/sanitize_run.py 2>&1 | tail -3; done
