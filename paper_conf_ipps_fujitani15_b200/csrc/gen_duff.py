@@ -269,7 +269,7 @@ def emit_cmpl(W: int, G: int, ones: bool) -> str:
     return "\n".join(o)
 
 
-def emit_hybrid(W: int, G: int, side: str) -> str:
+def emit_hybrid(W: int, G: int, side: str, form: str = "split") -> str:
     """Hybrid passes of the 4096-bit all-pairs kernel (kernels.cuh allpairs_hybrid_kernel):
     operand A lives in registers (top-aligned like every register kernel: word i at
     register s + i), operand B in shared memory, least significant word first, one row of
@@ -288,7 +288,7 @@ def emit_hybrid(W: int, G: int, side: str) -> str:
     sa = "%%%d" % (W + 3)
     ba = "%%%d" % (W + 4)
     K = lambda k: 128 * k
-    a = ["{", ".reg .u32 zp, z, lo, hi, t, v, w;", ".reg .u64 p, q;", ".reg .pred pe;",
+    a = ["{", ".reg .u32 zp, z, lo, hi, t, v, w;", ".reg .u64 p, q, m;", ".reg .pred pe;",
          "setp.ge.s32 pe, %s, 0;" % sa,
          "ts: .branchtargets %s;" % ", ".join("E%d" % k for k in range(W)),
          "brx.idx %s, ts;" % sa]
@@ -296,15 +296,20 @@ def emit_hybrid(W: int, G: int, side: str) -> str:
     def ldv(k):  # the shared-memory operand's word at register position k -> v
         return ["ld.shared.u32 v, [%s+%d];" % (ba, K(k))]
 
+    def product(k):  # p = alpha * (multiplicand word k) + carry, split or wide (emit's forms)
+        mw = "v" if side == "A" else av(k)
+        if form == "wide" or (form.startswith("mix") and k % int(form[3:]) != 0):
+            return ["mul.wide.u32 m, %s, %s;" % (al, mw), "shr.u64 q, p, 32;", "add.s64 p, m, q;",
+                    "mov.b64 {lo, hi}, p;"]
+        return ["mov.b64 q, {hi, 0};", "mad.wide.u32 p, %s, %s, q;" % (al, mw), "mov.b64 {lo, hi}, p;"]
+
     def limb(k):
-        out = ldv(k) + ["mov.b64 q, {hi, 0};"]
+        out = ldv(k) + product(k)
         if side == "A":
-            out += ["mad.wide.u32 p, %s, v, q;" % al, "mov.b64 {lo, hi}, p;",
-                    "subc.cc.u32 z, %s, lo;" % av(k),
+            out += ["subc.cc.u32 z, %s, lo;" % av(k),
                     "shf.r.wrap.b32 %s, zp, z, %%0;" % av(k - 1)]
         else:
-            out += ["mad.wide.u32 p, %s, %s, q;" % (al, av(k)), "mov.b64 {lo, hi}, p;",
-                    "subc.cc.u32 z, v, lo;",
+            out += ["subc.cc.u32 z, v, lo;",
                     "shf.r.wrap.b32 w, zp, z, %0;",
                     "st.shared.u32 [%s+%d], w;" % (ba, K(k - 1))]
         return out + ["mov.u32 zp, z;"]
@@ -362,6 +367,7 @@ def main():
     form = sys.argv[1] if len(sys.argv) > 1 else os.environ.get("BULKGCD_PASS_FORM", "mix2")
     form64 = os.environ.get("BULKGCD_PASS_FORM64", "split")
     formx = os.environ.get("BULKGCD_PASS_FORM_EXACT", "split")
+    formh = os.environ.get("BULKGCD_PASS_FORM_HYBRID", "split")  # 4096-bit hybrid passes
     G = int(os.environ.get("BULKGCD_PASS_G", "8" if form == "two" else "4"))
     # Exact-mode pairs kernel: G = 2 (cfg2 2^20 exact pairs 4.20 -> 3.87 ms; its larger
     # code -- Case-1 tail, L41 normalisation -- misses the i-cache at G = 4).  G = 2 for
@@ -415,8 +421,8 @@ def main():
         "__device__ __forceinline__ uint32_t duff_hpass(AR &A, uint32_t alpha, int s, uint32_t base, uint32_t &r);",
         "constexpr int PASS_G_HYBRID = %d;" % GH,
         "",
-        emit_hybrid(128, GH, "A"), "",
-        emit_hybrid(128, GH, "B"), "",
+        emit_hybrid(128, GH, "A", formh), "",
+        emit_hybrid(128, GH, "B", formh), "",
     ]
     for W in WIDTHS:
         gw = G64 if W >= 64 else (G16 if W <= 16 else G)
