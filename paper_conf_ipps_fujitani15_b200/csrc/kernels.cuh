@@ -169,7 +169,8 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // HOIST: approx() for the next iteration is computed at the end of the current one, ahead of
 // its votes and branches (measured: cfg4 851.5 -> 834.6 ms; cfg3 233.3 -> 235.1, 2^20 RSA pairs
 // 2.47 -> 3.07, exact 3.74 -> 3.84 ms: the W = 64 all-pairs kernel only).
-template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, bool CMPL = false, bool HOIST = false>
+template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, bool CMPL = false, bool HOIST = false,
+          bool SWAP_RESUME = false>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
@@ -257,6 +258,19 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
     for (;;) {
         bool more = resume == 0 ? cold(A, B, lA, tA, lB, tB) : cold(B, A, lB, tB, lA, tA);
         if (!more) return;
+        // SWAP_RESUME: resuming on roles (B, A) exchanges the register arrays (and their lengths
+        // and tops) instead, so the loop is entered at its first hot iteration only and the pass
+        // is inlined twice, with no irreducible entry: 64-128 moves on a cold exit (~1 % of the
+        // iterations) for a third less hot code (instruction cache).  In the complement form both
+        // arrays are complemented too, so that A stays the complemented one.
+        if (SWAP_RESUME && resume == 1) {
+            if (CMPL) cmpl_regs<W>(A);  // plain A0, B0
+            swap_regs<W>(A, B);
+            if (CMPL) cmpl_regs<W>(A);  // A = ~B0 (the complemented one again), B = A0
+            int tl = lA; lA = lB; lB = tl;
+            uint64_t tt = tA; tA = tB; tB = tt;
+            resume = 0;
+        }
         if (HOIST) ap = resume == 0 ? approx_pre<EXACT>(lA, tA, lB, tB) : approx_pre<EXACT>(lB, tB, lA, tA);
         // ONE_ENTRY: resuming on roles (B, A) enters the loop at its second hot
         // iteration, so the pass is inlined twice (once per role assignment) instead of
@@ -266,7 +280,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         // kernel uses it.
         if (ONE_ENTRY) {
             if (resume == 1) goto roles_ba;
-        } else if (resume == 1) {
+        } else if (!SWAP_RESUME && resume == 1) {
             if (hot(CmB{}, B, A, lB, tB, lA, tA)) {
                 resume = 0;
                 continue;
@@ -705,7 +719,9 @@ __global__ void BULKGCD_AP_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
         HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
-        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, allpairs_cmpl<W>(), (W >= 64)>(
+        // SWAP_RESUME: cfg3 233.3 -> 232.0 ms, cfg6 80.7 -> 79.2 ms, cfg4 834.8 -> 832.4 ms (the exact
+        // pairs kernel keeps three pass copies: with two, ptxas loses the uniform BRXU there, 3.74 -> 3.81 ms)
+        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, allpairs_cmpl<W>(), (W >= 64), true>(
             A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, 0, iters, nslow, limbs, slots, passw);
         slot ^= 1;
         have = have2;
