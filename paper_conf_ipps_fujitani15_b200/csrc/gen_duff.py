@@ -369,14 +369,17 @@ def main():
     formx = os.environ.get("BULKGCD_PASS_FORM_EXACT", "split")
     # 4096-bit hybrid passes: mix2 (cfg8 5,563 -> 5,219 ms, cfg7 5.9 -> 5.5 ms)
     formh = os.environ.get("BULKGCD_PASS_FORM_HYBRID", "mix2")
-    G = int(os.environ.get("BULKGCD_PASS_G", "8" if form == "two" else "4"))
+    # W = 32 blocks of 8 limbs once the all-pairs loop carried two pass copies (cfg3 231.7 -> 230.0 ms;
+    # 6: 230.8, 16: 271.9, 2: 240.7); W = 16 keeps 4 (its own knob below)
+    G = int(os.environ.get("BULKGCD_PASS_G", "8"))
     # Exact-mode pairs kernel: G = 2 (cfg2 2^20 exact pairs 4.20 -> 3.87 ms; its larger
     # code -- Case-1 tail, L41 normalisation -- misses the i-cache at G = 4).  G = 2 for
     # the all-pairs kernel costs 246.7 -> 250.7 ms on cfg3, G = 8: 247.3 ms (exact 4.99).
     # Exact at G = 1: 3.98 ms (2048-bit 3.74), G = 3: 4.00 ms (3.58), against 3.87 / 3.46 at G = 2.
     GX = int(os.environ.get("BULKGCD_PASS_G_EXACT", "2"))
     G64 = int(os.environ.get("BULKGCD_PASS_G64", "2"))  # W = 64 has its own knob
-    G16 = int(os.environ.get("BULKGCD_PASS_G16", str(G)))  # W = 16 at G = 2: cfg6 82.6 -> 83.4 ms (stays 4)
+    GR = int(os.environ.get("BULKGCD_PASS_G_RSA", "4"))  # RSA-mode pairs kernel, W <= 32
+    G16 = int(os.environ.get("BULKGCD_PASS_G16", "4"))  # W = 16 at G = 2: cfg6 82.6 -> 83.4 ms, 8: 79.1 -> 79.2
     here = os.path.dirname(os.path.abspath(__file__))
     fw = lambda W: form64 if W >= 64 else form
     parts = [
@@ -403,6 +406,9 @@ def main():
         "constexpr int PASS_G = W >= 64 ? %d : (W <= 16 ? %d : %d);" % (G64, G16, G),
         "template <int W>",
         "constexpr int PASS_F = W >= 64 ? %d : %d;  // %s / %s" % (form_code(form64), form_code(form), form64, form),
+        "// RSA-mode pairs kernel (one-entry loop): 4-limb blocks at W <= 32 (2^20 pairs 2.46 ms against 3.14 at 8)",
+        "template <int W>",
+        "constexpr int PASS_G_RSA = W >= 64 ? %d : %d;" % (G64, GR),
         "constexpr int PASS_G_EXACT = %d;  // exact-mode pairs kernel (smaller code: i-cache)" % GX,
         "constexpr int PASS_F_EXACT = %d;  // %s" % (form_code(formx), formx),
         "",
@@ -427,7 +433,8 @@ def main():
     ]
     for W in WIDTHS:
         gw = G64 if W >= 64 else (G16 if W <= 16 else G)
-        for g, f in sorted({(gw, fw(W)), (GX, formx)}):
+        gr = G64 if W >= 64 else GR
+        for g, f in sorted({(gw, fw(W)), (gr, fw(W)), (GX, formx)}):
             parts.append(emit_two(W, g) if f == "two" else emit(W, f, g))
             parts.append("")
         for ones in (True, False):

@@ -170,7 +170,7 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // its votes and branches (measured: cfg4 851.5 -> 834.6 ms; cfg3 233.3 -> 235.1, 2^20 RSA pairs
 // 2.47 -> 3.07, exact 3.74 -> 3.84 ms: the W = 64 all-pairs kernel only).
 template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, bool CMPL = false, bool HOIST = false,
-          bool SWAP_RESUME = false>
+          bool SWAP_RESUME = false, int PG = 0>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
@@ -228,7 +228,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         }
         bool full, post, lt;
         if (!HOIST) ap = approx_pre<EXACT>(lX, tX, lY, tY);
-        hot_iter<W, EXACT, decltype(cm)::value>(X, Y, lX, tX, lY, tY, s, live, ap, full, post, lt);
+        hot_iter<W, EXACT, decltype(cm)::value, PG>(X, Y, lX, tX, lY, tY, s, live, ap, full, post, lt);
         bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
         bool fin = live & !run & !bad;
@@ -464,8 +464,8 @@ __global__ void BULKGCD_BOUNDS(W, true) pairs_kernel(PairsArgs a) {
             PairsSinkRsa<W> sink{a.G, i, a.m_pad};
             // ONE_ENTRY (irreducible loop entry: the pass entry stays a per-thread BRX) beats the
             // two-entry loop with a uniform BRXU here: 2^20 RSA pairs 2.47 against 3.05 ms
-            euclid_loop<W, STATS, false, true>(A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, 0, iters, nslow, limbs,
-                                               slots, passw);
+            euclid_loop<W, STATS, false, true, RsaCond, PairsSinkRsa<W>, false, false, false, PASS_G_RSA<W>>(
+                A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, 0, iters, nslow, limbs, slots, passw);
         } else {
             int k2 = 0;
             bool known = false;
