@@ -18,6 +18,8 @@ JOBS = {  # workload -> (kernel regex, driver command)
     "cfg4": ("regex:allpairs_kernel", ["python", "tools/prof_allpairs.py", "cfg4", "1"]),
     "cfg6": ("regex:allpairs_kernel", ["python", "tools/prof_allpairs.py", "cfg6", "1"]),
     "cfg8": ("regex:allpairs_hybrid", ["python", "tools/prof_allpairs.py", "cfg8", "1"]),
+    # the 4096-bit hybrid kernel at cfg7 size (ncu fails to replay the 5.5 s cfg8 launch)
+    "cfg7": ("regex:allpairs_hybrid", ["python", "tools/prof_allpairs.py", "cfg7", "1"]),
     "cfg2": ("regex:pairs_kernel", ["python", "tools/prof_pairs.py", "1048576", "0"]),
 }
 

@@ -16,7 +16,7 @@ echo "algo/ref: $(cut -c1-120 $O/r2_bench_cfg3_algoC.json) | $(cut -c1-120 $O/r2
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/r2_launches.csv \
   python bench.py --steps 2 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $O/ncu_launch.log 2>&1; echo ncu_launch_rc=$?
 # one ncu --set full capture of the hot kernel per workload (roofline.traffic, stall mix)
-timeout 1800 python tools/ncu_traffic.py $O cfg3 cfg2 cfg4 cfg6 cfg8 > $O/traffic.log 2>&1; tail -5 $O/traffic.log
+timeout 1800 python tools/ncu_traffic.py $O cfg3 cfg2 cfg4 cfg6 cfg7 > $O/traffic.log 2>&1; tail -5 $O/traffic.log
 ncu -i $O/r2_cfg3.ncu-rep --page source --csv --print-source sass > $O/cfg3_src.csv 2>/dev/null
 ncu -i $O/r2_cfg3.ncu-rep --page raw --csv > $O/cfg3_raw.csv 2>/dev/null
 python tools/ncu_opmix.py $O/cfg3_src.csv > $O/r2_cfg3_opmix.txt 2>&1
