@@ -22,11 +22,9 @@ ncu -i $O/r2_cfg3.ncu-rep --page raw --csv > $O/cfg3_raw.csv 2>/dev/null
 python tools/ncu_opmix.py $O/cfg3_src.csv > $O/r2_cfg3_opmix.txt 2>&1
 # the reports themselves stay on the box (gpurun copies back at most 64 MiB)
 mkdir -p /tmp/ncu_reps && mv $O/*.ncu-rep /tmp/ncu_reps/ 2>/dev/null; gzip -f $O/cfg3_src.csv
-# compute-sanitizer on the same build
-{ echo "# compute-sanitizer on tools/sanitize_run.py (all-pairs at 512/1024/2048/4096 bits incl. the hybrid 4096-bit kernel, exact pairs on rare-path operands, the chunked two-stream host path); build $git_head"
-  for t in memcheck racecheck synccheck initcheck; do echo "== $t"; timeout 1200 compute-sanitizer --tool $t python tools/sanitize_run.py 2>&1 | tail -3; done
-} > $O/r2_compute_sanitizer.txt
-tail -12 $O/r2_compute_sanitizer.txt
+# compute-sanitizer is closed on this pool (profiles/r2_compute_sanitizer.txt): the same workload runs
+# plainly, checked against construction truth and math.gcd by its own asserts
+timeout 900 python tools/sanitize_run.py > $O/r2_sanitize_workload.txt 2>&1; echo "sanitize_run rc=$?" >> $O/r2_sanitize_workload.txt
 # microbenchmarks of the limb forms and pipes
 mkdir -p build
 nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o build/pipemix2 tools/pipemix2.cu && build/pipemix2 > $O/r2_pipemix2.json
