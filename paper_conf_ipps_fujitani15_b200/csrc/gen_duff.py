@@ -35,13 +35,11 @@ WIDTHS = (16, 32, 64)
 
 
 def form_code(form: str) -> int:
-    """duff_pass's third template argument: 0 split, 1 wide, M >= 2 mixM, 100 two-chain."""
+    """duff_pass's third template argument: 0 split, 1 wide, M >= 2 mixM."""
     if form == "split":
         return 0
     if form == "wide":
         return 1
-    if form == "two":
-        return 100
     assert form.startswith("mix") and int(form[3:]) >= 2, form
     return int(form[3:])
 
@@ -105,90 +103,6 @@ def emit(W: int, form: str = "split", G: int = 1) -> str:
         if k % G == 0:
             a.append("B%d:" % k)
         a += limb(k)
-    a += ["TOP:", "shf.r.wrap.b32 %s, zp, 0, %%0;" % xa(W - 1), "}"]
-    body = "\\n\\t".join(x.replace('"', '\\"') for x in a)
-    outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(X[%d])' % k for k in range(W)]
-    ins = ['"r"(Y[%d])' % k for k in range(W)] + ['"r"(alpha)', '"r"(s)']
-    o = ["template <>",
-         "__device__ __forceinline__ uint32_t duff_pass<%d, %d, %d>(uint32_t (&X)[%d], const uint32_t (&Y)[%d], "
-         "uint32_t alpha, int s, uint32_t &r) {" % (W, G, FCODE, W, W),
-         "  uint32_t zs;",
-         '  asm volatile("%s"' % body,
-         "      : %s" % ", ".join(outs),
-         "      : %s);" % ", ".join(ins),
-         "  return zs;",
-         "}"]
-    return "\n".join(o)
-
-
-def emit_two(W: int, G: int) -> str:
-    """Two-borrow-chain form: Z = X - lo(alpha*Y) - hi(alpha*Y)*D, per G-limb block
-    chain 1 subtracts the low product words, chain 2 the high words one limb up
-    (tools/limbmix.cu: no carry-add / IMAD.X per limb; 9.5 -> 8.9 SMSP-cycles per
-    limb in isolation at G = 8).  The borrows cross block boundaries through two
-    registers (save: subc 0,0 -> 0 or -1; restore: sub.cc 0, b)."""
-    FCODE = form_code("two")
-    xa = lambda k: "%%%d" % (2 + k)
-    ya = lambda k: "%%%d" % (W + 2 + k)
-    al = "%%%d" % (2 * W + 2)
-    sa = "%%%d" % (2 * W + 3)
-    regs = ", ".join([f"l{g}, h{g}, z{g}" for g in range(G)])
-    a = ["{", f".reg .u32 zp, hp, b1, b2, t, {regs};", ".reg .u64 p;", ".reg .pred pe;",
-         "setp.ge.s32 pe, %s, 0;" % sa,
-         "ts: .branchtargets %s;" % ", ".join("E%d" % k for k in range(W)),
-         "brx.idx %s, ts;" % sa]
-
-    def block(k0, k1, head):
-        """limbs k0..k1-1 (one G-block or the head's partial block)."""
-        n = k1 - k0
-        out = []
-        for g in range(n):
-            out += ["mul.wide.u32 p, %s, %s;" % (al, ya(k0 + g)), f"mov.b64 {{l{g}, h{g}}}, p;"]
-        # chain 1: z = x - lo
-        if head:
-            out.append("sub.cc.u32 z0, %s, l0;" % xa(k0))
-        else:
-            out += ["sub.cc.u32 t, 0, b1;", "subc.cc.u32 z0, %s, l0;" % xa(k0)]
-        for g in range(1, n):
-            out.append(f"subc.cc.u32 z{g}, %s, l{g};" % xa(k0 + g))
-        out.append("subc.u32 b1, 0, 0;")
-        if head:  # r = ctz(z_s): chain 2 does not touch the first limb
-            out += ["mov.u32 %1, z0;", "brev.b32 t, z0;", "clz.b32 %0, t;"]
-        # chain 2: z -= hi one limb up (hp = hi of the limb below the block)
-        if head:
-            if n > 1:
-                out.append("sub.cc.u32 z1, z1, h0;")
-                for g in range(2, n):
-                    out.append(f"subc.cc.u32 z{g}, z{g}, h{g - 1};")
-                out.append("subc.u32 b2, 0, 0;")
-            else:
-                out.append("mov.u32 b2, 0;")
-        else:
-            out += ["sub.cc.u32 t, 0, b2;", "subc.cc.u32 z0, z0, hp;"]
-            for g in range(1, n):
-                out.append(f"subc.cc.u32 z{g}, z{g}, h{g - 1};")
-            out.append("subc.u32 b2, 0, 0;")
-        out.append(f"mov.u32 hp, h{n - 1};")
-        # funnel shifts: X[k-1] = (z_{k-1}, z_k) >> r
-        for g in range(n):
-            k = k0 + g
-            if head and g == 0:
-                pass
-            else:
-                out.append(f"shf.r.wrap.b32 %s, zp, z{g}, %%0;" % xa(k - 1))
-            out.append(f"mov.u32 zp, z{g};")
-        return out
-
-    for k in range(W):
-        e = min((k // G + 1) * G, W)
-        nxt = "B%d" % e if e < W else "TOP"
-        a.append("E%d:" % k)
-        a += block(k, e, True)
-        a.append("@pe bra %s;" % nxt)
-    a.append("bra.uni TOP;")
-    for k in range(G, W, G):
-        a.append("B%d:" % k)
-        a += block(k, min(k + G, W), False)
     a += ["TOP:", "shf.r.wrap.b32 %s, zp, 0, %%0;" % xa(W - 1), "}"]
     body = "\\n\\t".join(x.replace('"', '\\"') for x in a)
     outs = ['"=r"(r)', '"=r"(zs)'] + ['"+r"(X[%d])' % k for k in range(W)]
@@ -395,7 +309,7 @@ def main():
         "// Returns z_s (the lowest word of X - alpha*Y); r = ctz(z_s) (32 if z_s == 0, in which",
         "// case the funnel shifts wrap to 0 and X holds X - alpha*Y unshifted).",
         "// G = limbs per straight-line block of the chain (one predicated branch per block);",
-        "// F = limb form (gen_duff.form_code: 0 split, 1 wide, M >= 2 every M-th limb split, 100 two-chain).",
+        "// F = limb form (gen_duff.form_code: 0 split, 1 wide, M >= 2 every M-th limb split).",
         "template <int W, int G, int F>",
         "__device__ __forceinline__ uint32_t duff_pass(uint32_t (&X)[W], const uint32_t (&Y)[W], uint32_t alpha, int s,",
         "                                              uint32_t &r);",
@@ -435,7 +349,7 @@ def main():
         gw = G64 if W >= 64 else (G16 if W <= 16 else G)
         gr = G64 if W >= 64 else GR
         for g, f in sorted({(gw, fw(W)), (gr, fw(W)), (GX, formx)}):
-            parts.append(emit_two(W, g) if f == "two" else emit(W, f, g))
+            parts.append(emit(W, f, g))
             parts.append("")
         for ones in (True, False):
             parts.append(emit_cmpl(W, gw, ones))
