@@ -663,7 +663,8 @@ def main():
             "roofline": roofline(limbs / world, iters / world, pairs / world, kern_s, sms,
                                  (f"allpairs_kernel<{W}>" if W < 128 else f"allpairs_hybrid_kernel<{W}>")
                                  if args.algo == "E" else f"allpairs_*_kernel<{W}, {args.algo}>",
-                                 kern_total_ms / step_total_ms, _traffic(args.workload), eff),
+                                 kern_total_ms / step_total_ms,
+                                 _traffic(args.workload) if args.algo == "E" else None, eff),
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(Nh.nbytes) * world,
                     "d2h_bytes_per_step": int(d2h) * world} if e2e_value else None,
             "gpu_launches": 2 * args.steps,

@@ -201,6 +201,21 @@ def test_all_pairs_stats_counters(bg, cfg1):
     assert int(ctr[4]) == sum(t.limb_steps for t in tr)      # limb-steps (the roofline's unit, M2)
 
 
+@pytest.mark.parametrize("bits,n", [(512, 72), (2048, 40)])
+def test_all_pairs_stats_counters_widths(bg, bits, n):
+    """Per-width iteration and limb-step totals of the all-pairs kernels (W = 16: 4-limb mix2 pass;
+    W = 64: complement form, approx() hoisted, swap on resume) equal the paper's algorithm as the
+    model runs it (L107/L127, RSA mode), with planted hits and a clique among the moduli."""
+    ms = synth.moduli(n, bits, seed=7000 + bits, n_planted_pairs=3, cliques=(3,))
+    total = bg.bulkgcd_cohort_count(ms.m)
+    count, out, ctr = _band_run(bg, ms, bits, 0, total, 64)
+    assert out == ms.truth and count == len(ms.truth)
+    N = synth.ints(ms.N)
+    tr = [am.gcd_rsa(N[i], N[j], bits) for i in range(n) for j in range(i + 1, n)]
+    assert int(ctr[2]) == sum(t.iterations for t in tr)
+    assert int(ctr[4]) == sum(t.limb_steps for t in tr)
+
+
 def _golden_hits(name):
     """(sha256 of N, sorted [(i, j, g)]) from a tools/oracle_sweep.py golden file."""
     import os
