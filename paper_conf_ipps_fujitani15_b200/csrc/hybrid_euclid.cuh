@@ -208,11 +208,14 @@ __device__ __forceinline__ void hybrid_loop(uint32_t (&A)[W], uint32_t bbase, in
     for (;;) {
         bool more = resume == 0 ? cold(false, lA, tA, lB, tB) : cold(true, lB, tB, lA, tA);
         if (!more) return;
+        // Resuming with B updated next: exchange the operands (registers <-> shared memory) instead
+        // of entering the loop at its second iteration, so the pass is inlined twice, not three
+        // times (instruction cache; as euclid_loop's SWAP_RESUME).
         if (resume == 1) {
-            if (hot(SB{}, lB, tB, lA, tA)) {
-                resume = 0;
-                continue;
-            }
+            h_swap<W>(A, base(), s);
+            int tl = lA; lA = lB; lB = tl;
+            uint64_t tt = tA; tA = tB; tB = tt;
+            resume = 0;
         }
         for (;;) {
             if (hot(SA{}, lA, tA, lB, tB)) {

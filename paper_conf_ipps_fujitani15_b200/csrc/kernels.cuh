@@ -30,6 +30,9 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 // 24 warps 4.32 / 3.47 ms
 #define MIN_WARPS_PAIRS 20
 #endif
+#ifndef MIN_WARPS_W16_PAIRS
+#define MIN_WARPS_W16_PAIRS 32  // 512-bit pairs: 2^20 exact 1.49 -> 1.46 ms, RSA 0.85 -> 0.83 ms against 20
+#endif
 #ifndef MIN_WARPS_W64
 // W = 64 all-pairs: 12 warps/SM (168 registers; ptxas spills ~4 KB of cold and window state)
 // beat 8 warps (255 registers, spill-free): cfg4 1,034 -> 943 ms; 16 warps spill the
@@ -51,7 +54,8 @@ constexpr int WARPS_PER_CTA = THREADS / 32;
 template <int W, bool PAIRS = false>
 struct Occ {
     static constexpr int warps = W >= 64 ? (PAIRS ? MIN_WARPS_W64_PAIRS : MIN_WARPS_W64)
-                                         : (PAIRS ? MIN_WARPS_PAIRS : (W <= 16 ? MIN_WARPS_W16 : MIN_WARPS));
+                                         : (PAIRS ? (W <= 16 ? MIN_WARPS_W16_PAIRS : MIN_WARPS_PAIRS)
+                                                  : (W <= 16 ? MIN_WARPS_W16 : MIN_WARPS));
     static constexpr int blocks = warps / WARPS_PER_CTA > 0 ? warps / WARPS_PER_CTA : 1;
 };
 
