@@ -343,6 +343,43 @@ def test_distributed_band_driver_on_one_gpu(bg):
     assert all(out[r][0] for r in range(3)), dict(out)
 
 
+def _nccl_worker(rank, world, port, out):
+    import os
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    dist.init_process_group("nccl", rank=rank, world_size=world, device_id=dev)
+    from paper_conf_ipps_fujitani15_b200 import dist as bgd
+    ms = synth.moduli(200, 1024, seed=78, n_planted_pairs=5, cliques=(3,))
+    N = torch.from_numpy(ms.N.view(np.int32)).to(dev)
+    dist.broadcast(N, src=0)  # bench.py's replication of the moduli (rank 0 generates)
+    st = bgd.AllPairsBand(N.cpu().numpy().view(np.uint32), 1024, rank, world)
+    st.upload()
+    st.layout()
+    st.search()
+    rec = bgd.gather_hits(st.local_hits())  # NCCL all-gather of counts + padded records
+    hits = bgd.records_to_hits(rec.cpu().numpy(), 1024).as_list()
+    out[rank] = (hits == ms.truth, len(hits), dist.get_backend(), rec.is_cuda)
+    dist.destroy_process_group()
+
+
+def test_nccl_exchange_single_rank(bg):
+    """The NCCL data plane of the multi-GPU path (communicator on cuda:0, broadcast of the
+    moduli, all-gather of hit counts and padded hit records on device tensors) with one rank:
+    the only NCCL configuration a one-GPU box can run without ranks that wait on each other."""
+    import socket
+    import torch.multiprocessing as mp
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    out = mp.Manager().dict()
+    mp.spawn(_nccl_worker, args=(1, port, out), nprocs=1, join=True)
+    ok, n, backend, on_device = out[0]
+    assert ok and backend == "nccl" and on_device, dict(out)
+
+
 def test_bench_multirank_path_gloo(bg):
     """bench.py's N > 1 code path (torchrun, band split, hit exchange, max-over-ranks
     timing) on the single test GPU, with gloo standing in for NCCL."""
