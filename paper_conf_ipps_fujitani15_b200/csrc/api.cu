@@ -221,7 +221,7 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
                     uint64_t cap, unsigned long long *counters, unsigned flags, cudaStream_t st) {
     CK(cudaMemsetAsync(counters, 0, 8 * sizeof(unsigned long long), st));
     if (c1 <= c0) return 0;
-    AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16};
+    AllPairsArgs a{dBlk, dN, n, c0, c1, counters + 1, dHits, cap, counters, counters + 2, W * 16, nullptr};
     if constexpr (W >= 128) {
         // the 4096-bit product path: the hybrid kernel (A in registers, B in shared memory);
         // BULKGCD_FLAG_SMEM and the comparison algorithms keep the shared-memory kernels
@@ -267,6 +267,12 @@ int launch_allpairs(const uint32_t *dN, const uint32_t *dBlk, size_t n, uint64_t
             return 0;
         }))
         return rc;
+    // straggler buffers (allpairs_cutk): one per resident warp, from the device's default pool
+    DBuf strag;
+    if constexpr (allpairs_cutk<W>() > 0) {
+        CK(strag.alloc(grid * ApCfg<W>::warps_per_cta * strag_words<W>() * STRAG_CAP * sizeof(uint32_t), st));
+        a.strag = strag.as<uint32_t>();
+    }
     if (flags & BULKGCD_FLAG_STATS) allpairs_kernel<W, true><<<(unsigned)grid, ApCfg<W>::threads, smem, st>>>(a);
     else allpairs_kernel<W, false><<<(unsigned)grid, ApCfg<W>::threads, smem, st>>>(a);
     CK(cudaGetLastError());

@@ -173,8 +173,12 @@ __device__ __forceinline__ void setup_pair(uint32_t (&A)[W], uint32_t (&B)[W], i
 // HOIST: approx() for the next iteration is computed at the end of the current one, ahead of
 // its votes and branches (measured: cfg4 851.5 -> 834.6 ms; cfg3 233.3 -> 235.1, 2^20 RSA pairs
 // 2.47 -> 3.07, exact 3.74 -> 3.84 ms: the W = 64 all-pairs kernel only).
+// CUTK > 0: straggler cut (all-pairs, split/mix forms only).  Every second iteration the warp counts
+// its running lanes; once at most CUTK remain, sink.cut() stores their operands (and pair ids) in the
+// warp's straggler buffer and the cohort ends; the kernel runs the stored lanes later, 32 at a time
+// (allpairs_kernel), so the end of a cohort no longer runs a nearly empty warp.
 template <int W, bool STATS, bool EXACT, bool ONE_ENTRY, class Cond, class Sink, bool CMPL = false, bool HOIST = false,
-          bool SWAP_RESUME = false, int PG = 0>
+          bool SWAP_RESUME = false, int PG = 0, int CUTK = 0>
 __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], int &lA, uint64_t &tA, int &lB,
                                             uint64_t &tB, bool live, Cond cond, Sink &sink, int s0,
                                             uint32_t &iters, uint32_t &nslow, uint32_t &limbs, uint32_t &slots,
@@ -221,6 +225,7 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
     // One hot iteration on roles (X, Y) (its loop test already passed: the
     // live lanes are the running ones), then the loop test of the next
     // iteration (roles (Y, X)).  Returns true to go cold.
+    bool cut = false;
     auto hot = [&](auto cm, uint32_t(&X)[W], uint32_t(&Y)[W], int &lX, uint64_t &tX, int &lY, uint64_t &tY) -> bool {
         if (STATS) {
             ++slots;
@@ -244,6 +249,15 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
         if (any_need) {
             fix = fix_code(live, full, post, lt);
             return true;
+        }
+        if constexpr (CUTK > 0) {
+            if (decltype(cm)::value == 0 && &X == &B) {  // after the B-updating iteration only
+                if (__popc(__ballot_sync(FULL, run)) <= sink.cutk) {
+                    live = run;
+                    cut = true;
+                    return true;
+                }
+            }
         }
         if (!any_top) {  // the warp length dropped (lanes finished or shrank): realign one word in place
             unsigned brun = __ballot_sync(FULL, run);
@@ -299,6 +313,12 @@ __device__ __forceinline__ void euclid_loop(uint32_t (&A)[W], uint32_t (&B)[W], 
             if (hot(CmB{}, B, A, lB, tB, lA, tA)) {
                 resume = 0;
                 break;
+            }
+        }
+        if constexpr (CUTK > 0) {
+            if (cut) {  // the last iteration updated B and went through no fix-up: A >= B
+                sink.cut(live, A, B, s, lA);
+                return;
             }
         }
     }
@@ -544,7 +564,15 @@ struct AllPairsArgs {
     unsigned long long *hit_count;
     unsigned long long *stats;     // optional [sum iterations, slow steps, limb-steps]
     int half;
+    uint32_t *strag;               // straggler buffers, one per resident warp (W <= 32)
 };
+
+// Straggler buffer of one warp (euclid_loop's CUTK): STRAG_CAP records of (i, j, length, A[W], B[W])
+// with the numbers least significant word first (not top-aligned), word-major: record r's word k at
+// rec[k * STRAG_CAP + r], so the lanes of a warp store and load consecutive words.
+constexpr int STRAG_CAP = 64;
+template <int W>
+__host__ __device__ constexpr int strag_words() { return 3 + 2 * W; }
 
 template <int W>
 struct HitSink {
@@ -552,6 +580,30 @@ struct HitSink {
     uint64_t cap;
     unsigned long long *count;
     uint32_t i, j;
+    uint32_t *strag = nullptr;  // this warp's straggler buffer (CUTK)
+    int *nstrag = nullptr;      // its fill level (warp-uniform)
+    int cutk = -1;              // cut when at most cutk lanes still run (-1: never)
+    // Store the running lanes' pairs (registers top-aligned at the warp-uniform s; word k of a
+    // number in register s + k) least significant word first, with A's length lA (A >= B).
+    __device__ __forceinline__ void cut(bool run, const uint32_t (&A)[W], const uint32_t (&B)[W], int s, int lA) {
+        const int lane = threadIdx.x & 31;
+        unsigned b = __ballot_sync(FULL, run);
+        int slot = *nstrag + __popc(b & ((1u << lane) - 1u));
+        if (run) {
+            uint32_t *r = strag + slot;
+            r[0] = i;
+            r[STRAG_CAP] = j;
+            r[2 * STRAG_CAP] = (uint32_t)lA;
+#pragma unroll
+            for (int k = 0; k < W; ++k) {
+                if (k >= s) {
+                    r[(3 + k - s) * STRAG_CAP] = A[k];
+                    r[(3 + W + k - s) * STRAG_CAP] = B[k];
+                }
+            }
+        }
+        *nstrag += __popc(b);
+    }
     // a lane that stops with Y != 0 is coprime-mode ("return 1", L243/L251): nothing to report
     __device__ __forceinline__ bool quick(bool fin, int, uint64_t, int lY, uint64_t) { return fin && lY == 0; }
     // In the hot loop a lane only finishes with Y = X' != 0 (a zero X' sets `post` and goes cold):
@@ -664,6 +716,14 @@ __device__ __forceinline__ void cohort_coords(uint64_t c, uint64_t n, uint64_t &
 template <int W>
 __host__ __device__ constexpr bool allpairs_cmpl() { return W >= BULKGCD_ALLPAIRS_CMPL_MIN_W; }
 
+// Straggler cut threshold of the all-pairs kernel by width (0: off; never with the complement form).
+// Measured (cfg6 / cfg3): W = 16 79.2 -> 77.5 ms at 8, 77.3 ms at 12 (lane efficiency 0.870 -> 0.951);
+// W = 32 229.5 -> 240.9 / 255.2 / 270.1 ms at 4 / 8 / 12 although warp-iterations drop 5 %: a batch
+// mixes lanes of different cohorts and lengths, whose tops fall below the 5-register window (slow
+// steps and window misses per pair 0.020 -> 0.063 at 8), and every such cold exit spills the state.
+template <int W>
+__host__ __device__ constexpr int allpairs_cutk() { return W <= 16 ? 12 : 0; }
+
 #ifdef BULKGCD_MAXNREG
 #define BULKGCD_AP_BOUNDS(W) __maxnreg__(BULKGCD_MAXNREG)
 #else
@@ -702,36 +762,82 @@ __global__ void BULKGCD_AP_BOUNDS(W) allpairs_kernel(AllPairsArgs a) {
         return true;
     };
 
+    // Straggler cut (euclid_loop's CUTK), W <= 32: this warp's buffer and fill level
+    constexpr int kCutMax = allpairs_cutk<W>();
+    const int kCut = a.strag ? kCutMax : -1;
+    uint32_t *my_strag =
+        a.strag ? a.strag + ((uint64_t)blockIdx.x * ApCfg<W>::warps_per_cta + warp) * strag_words<W>() * STRAG_CAP
+                : nullptr;
+    int nstrag = 0;
+
+    // One work item per trip -- a cohort, or 32 stored stragglers once the buffer holds a full warp
+    // of them (and at the end, whatever is left, run to completion) -- through a single inlined
+    // euclid_loop (instruction cache).
     int slot = 0;
     uint64_t c, b, j;
     bool have = claim(0, c, b, j);
-    while (have) {
-        uint64_t c2, b2, j2;
-        bool have2 = claim(slot ^ 1, c2, b2, j2);  // prefetch the next cohort
-        mbar_wait(&bar[slot], phase[slot]);
-        phase[slot] ^= 1;
-        uint64_t i = 32 * b + lane;
-        bool live = i < j;
-        uint32_t A[W], B[W];
-#pragma unroll
-        for (int k = 0; k < W; ++k) {
-            A[k] = buf[slot].row[k * 32 + lane];  // conflict-free: one bank per lane
-            B[k] = buf[slot].col[k];              // broadcast
+    for (;;) {
+        int cnt = 0, cutk = kCut;
+        if (kCutMax > 0 && nstrag >= 32) {
+            cnt = 32;
+        } else if (!have) {
+            if (nstrag == 0) break;
+            cnt = nstrag;  // < 32: the last batch, no further cut
+            cutk = -1;
         }
-        __syncwarp();  // the buffer is refilled only after the next claim, i.e. after this read
+        uint32_t A[W], B[W];
+        bool live;
+        uint32_t ri, rj;
+        int s0 = 0;
+        uint64_t c2 = 0, b2 = 0, j2 = 0;
+        bool have2 = false;
+        if (cnt == 0) {  // the next cohort: its operands were staged by TMA
+            have2 = claim(slot ^ 1, c2, b2, j2);  // prefetch the one after
+            mbar_wait(&bar[slot], phase[slot]);
+            phase[slot] ^= 1;
+            uint64_t i = 32 * b + lane;
+            live = i < j;
+            ri = (uint32_t)i;
+            rj = (uint32_t)j;
+#pragma unroll
+            for (int k = 0; k < W; ++k) {
+                A[k] = buf[slot].row[k * 32 + lane];  // conflict-free: one bank per lane
+                B[k] = buf[slot].col[k];              // broadcast
+            }
+            __syncwarp();  // the buffer is refilled only after the next claim, i.e. after this read
+        } else {  // stored stragglers (the top of the buffer), loaded top-aligned at their longest length
+            nstrag -= cnt;
+            const uint32_t *r = my_strag + nstrag + lane;
+            live = lane < cnt;
+            ri = live ? r[0] : 0u;
+            rj = live ? r[STRAG_CAP] : 0u;
+            int rl = live ? (int)r[2 * STRAG_CAP] : 0;
+            s0 = W - (int)__reduce_max_sync(FULL, (unsigned)rl);
+#pragma unroll
+            for (int k = 0; k < W; ++k) {
+                int q = k - s0;  // word q of the numbers sits in register s0 + q
+                bool in = (q >= 0) & (q < rl);
+                A[k] = in ? r[(3 + q) * STRAG_CAP] : 0u;
+                B[k] = in ? r[(3 + W + q) * STRAG_CAP] : 0u;
+            }
+        }
         int lA, lB;
         uint64_t tA, tB;
         setup_pair<W>(A, B, lA, tA, lB, tB);
-        HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, (uint32_t)i, (uint32_t)j};
+        lA = lA > 0 ? lA - s0 : 0;  // lengths count from the start register s0
+        lB = lB > 0 ? lB - s0 : 0;
+        HitSink<W> sink{a.hits, a.hit_cap, a.hit_count, ri, rj, my_strag, &nstrag, cutk};
         // SWAP_RESUME: cfg3 233.3 -> 232.0 ms, cfg6 80.7 -> 79.2 ms, cfg4 834.8 -> 832.4 ms (the exact
         // pairs kernel keeps three pass copies: with two, ptxas loses the uniform BRXU there, 3.74 -> 3.81 ms)
-        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, allpairs_cmpl<W>(), (W >= 64), true>(
-            A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, 0, iters, nslow, limbs, slots, passw);
-        slot ^= 1;
-        have = have2;
-        c = c2;
-        b = b2;
-        j = j2;
+        euclid_loop<W, STATS, false, false, RsaCond, HitSink<W>, allpairs_cmpl<W>(), (W >= 64), true, 0, kCutMax>(
+            A, B, lA, tA, lB, tB, live, RsaCond{a.half}, sink, s0, iters, nslow, limbs, slots, passw);
+        if (cnt == 0) {
+            slot ^= 1;
+            have = have2;
+            c = c2;
+            b = b2;
+            j = j2;
+        }
     }
     if (STATS && a.stats) {
         atomicAdd(&a.stats[0], (unsigned long long)iters);
