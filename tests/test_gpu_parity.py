@@ -300,7 +300,7 @@ def test_pairs_config2_full_rsa_mode(bg):
 
 
 def test_pairs_chunked_host_path(bg):
-    """Host batches above 2^18 pairs run in overlapped chunks on two streams:
+    """Host batches above 2^17 pairs run in overlapped chunks on three streams:
     gcds and per-pair iteration counts equal single-chunk calls on the same
     pairs (ragged last chunk, both modes), and the gcds equal the oracle on a
     sample."""
@@ -409,7 +409,7 @@ def test_bench_multirank_path_gloo(bg):
 def test_concurrent_host_threads(bg, cfg1):
     """include/bulkgcd.h B5 (reentrant; the only global state is the lazily created
     per-device context): 4 host threads call bulkgcd_pairs (one of them above the
-    2^18-pair chunk size, i.e. the two-stream chunked path) and bulkgcd_all_pairs at
+    2^17-pair chunk size, i.e. the multi-stream chunked path) and bulkgcd_all_pairs at
     the same time, three rounds each.  ctypes drops the GIL around the C calls, so the
     calls overlap; every result must equal the oracle's."""
     import threading
