@@ -41,21 +41,14 @@ constexpr int HWIN = 12;  // top window of the 4096-bit operands (the wider spre
 // One hot iteration of the hybrid loop: SIDE 'A' updates A (registers) with multiplicand B
 // (shared memory), SIDE 'B' updates B with multiplicand A.  (lX, tX) are the updated
 // operand's cached length and top pair, (lY, tY) the multiplicand's; as hot_iter<W, false>.
+// `ap` = approx_pre<false>(lX, tX, lY, tY) (euclid.cuh: L127 Case 4, the exact floor, the odd alpha of
+// L107), computed by the loop at the end of the previous iteration (hoisted ahead of its votes).
 template <int W, char SIDE>
 __device__ __forceinline__ void hot_iter_h(uint32_t (&A)[W], uint32_t base, int &lX, uint64_t &tX, int lY,
-                                           uint64_t tY, int s, bool run, bool &full, bool &post, bool &lt) {
-    bool c4a = tX > tY;                                    // <x1x2> > <y1y2>        (L127, Case 4-A)
-    int d = lX - lY;
-    uint64_t den = (c4a ? tY : (uint64_t)hi32(tY)) + 1;    // 4-A: <y1y2>+1, 4-B: y1+1
-    bool near;
-    uint32_t qhi;
-    uint32_t q = div_floor_est(tX, den, near, qhi);
-    bool c4c = !c4a & (d == 0);
-    bool betapos = d > (c4a ? 0 : 1);
-    uint32_t alpha = c4c ? 1u : q;
-    alpha -= ~alpha & 1u;                                  // alpha is odd (L107)
-    full = betapos | (near & !c4c);
-    alpha = (run & !full) ? alpha : 0u;                    // the pass is a no-op for every other lane
+                                           uint64_t tY, int s, bool run, const Approx &ap, bool &full, bool &post,
+                                           bool &lt) {
+    full = ap.full;
+    uint32_t alpha = (run & !full) ? ap.a : 0u;           // the pass is a no-op for every other lane
     uint32_t r;
     uint32_t zs = duff_hpass<W, PASS_G_HYBRID, SIDE>(A, alpha, s, base, r);
     uint64_t t;
@@ -133,6 +126,7 @@ __device__ __forceinline__ void hybrid_loop(uint32_t (&A)[W], uint32_t bbase, in
     int s = 0;
     int fix = 0;     // pending fix-up of the last iteration (fix_code)
     int resume = 0;  // roles of the next iteration: 0 -> A updated (X = A), 1 -> B updated
+    Approx ap;       // approx() for the coming hot iteration
     auto base = [&]() { return bbase - 128u * (uint32_t)s; };
 
     // Cold section for the next roles; xb: X (the operand updated next) is B.
@@ -180,12 +174,13 @@ __device__ __forceinline__ void hybrid_loop(uint32_t (&A)[W], uint32_t bbase, in
             }
         }
         bool full, post, lt;
-        hot_iter_h<W, SIDE>(A, base(), lX, tX, lY, tY, s, live, full, post, lt);
+        hot_iter_h<W, SIDE>(A, base(), lX, tX, lY, tY, s, live, ap, full, post, lt);
         bool bad = live & (full | post | !lt);
         bool run = live & cond(lY, tY, lX, tX);
         bool fin = live & !run & !bad;
         bool need = sink.quick_hot(fin, lY, tY, lX, tX) | bad;
         bool top = run & (lY == W - s);
+        ap = approx_pre<false>(lY, tY, lX, tX);  // the next iteration's roles, ahead of the votes
         bool any_need = __any_sync(FULL, need), any_top = __any_sync(FULL, top);
         if (any_need) {
             fix = fix_code(live, full, post, lt);
@@ -217,6 +212,7 @@ __device__ __forceinline__ void hybrid_loop(uint32_t (&A)[W], uint32_t bbase, in
             uint64_t tt = tA; tA = tB; tB = tt;
             resume = 0;
         }
+        ap = approx_pre<false>(lA, tA, lB, tB);
         for (;;) {
             if (hot(SA{}, lA, tA, lB, tB)) {
                 resume = 1;
