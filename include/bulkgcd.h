@@ -161,7 +161,9 @@ int bulkgcd_pairs_device(const uint32_t *d_A, const uint32_t *d_B, uint32_t *d_G
  * is the SIMT lane efficiency), [6] = lane-words issued by the passes ([4]/[6]
  * is the pass-word efficiency); the shared-memory kernels as for
  * bulkgcd_pairs_device, with [7] = iterations with beta > 0 (L253).  Moduli
- * must be odd and > 1 (not checked here).
+ * must be odd and > 1 (not checked here).  At 512 bits the call also takes a
+ * stream-ordered scratch buffer from the device's default pool for the
+ * kernel's straggler cut (~42 MiB, released on `stream` after the launch).
  */
 int bulkgcd_all_pairs_band(const uint32_t *d_N, const uint32_t *d_N_blk, size_t n, uint32_t bits,
                            uint64_t cohort_begin, uint64_t cohort_end, uint32_t *d_hits, uint64_t hit_cap,
